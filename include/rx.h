@@ -1,0 +1,139 @@
+/*
+ * rx.h -- C ABI of the B200-native interleaved bitstream regex engine.
+ *
+ * The operation (PAPER.md = /root/reference/PAPER.md; "P:Lnnn" = its line):
+ *   a set of regular expressions is "evaluated concurrently over a shared
+ *   input stream" (Sec. 3.1); for each regex r the result is the
+ *   match-end bitstream S_r, "a 1 at position i indicates a successful match
+ *   ending at that position" under all-match semantics (Sec. 2), plus
+ *   per-regex match counts (the paper validates "match positions and counts",
+ *   P:L401).  Precisely: S_r[i] = 1 iff some s <= i has input[s..i] in L(r)
+ *   (non-empty, unanchored; DESIGN.md "Readings" c1-c17).
+ *
+ * How: rx_compile lowers patterns to a Parabix-style bitstream IR
+ * (CC from 8 basis streams, AND/OR/NOT, Advance, MatchStar, while -- Fig. 2,
+ * P:L77-116; Listing 3), groups regexes and
+ * JIT-compiles one fused interleaved sm_100a kernel (Sec. 3.3)
+ * with NVRTC.  rx_match launches it; no CPU fallback exists -- every
+ * function that computes returns RX_ECUDA when no CUDA device is usable.
+ *
+ * Conventions
+ *  - All pointers named d_* are DEVICE pointers (cudaMalloc / torch CUDA
+ *    tensors).  The caller owns the input and every output buffer; the
+ *    library owns the program and its scratch (stream-ordered).
+ *  - Calls that take a stream are asynchronous: they return a launch status;
+ *    device-side conditions are reported in out->d_status.
+ *  - Positions are 64-bit (inputs may exceed 2^32 bytes).
+ *  - Thread safety: distinct (rx_program, stream) pairs may be used
+ *    concurrently from different host threads.
+ */
+#ifndef RX_H_
+#define RX_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct rx_program rx_program; /* opaque: host IR + loaded sm_100a module */
+
+typedef enum {
+  RX_OK = 0,
+  RX_EPARSE = 1,       /* pattern syntax error (err->pattern_index / byte_offset) */
+  RX_EUNSUPPORTED = 2, /* anchors, backreferences, lookaround, lazy quantifiers */
+  RX_ETOOBIG = 3,      /* expansion of R{n,m} or program size over the caps */
+  RX_EJIT = 4,         /* NVRTC / module load failure (err->msg has the log head) */
+  RX_ECUDA = 5,        /* CUDA runtime error or no usable device */
+  RX_EINVAL = 6,       /* bad argument (NULL, misaligned, too small) */
+  RX_ENOMEM = 7,
+  RX_EOVERFLOW = 8
+} rx_status;
+
+typedef struct {
+  uint32_t pattern_index; /* which pattern failed */
+  uint32_t byte_offset;   /* where in it */
+  char msg[256];
+} rx_error;
+
+/* Tunables.  Defaults follow the paper's fixed defaults (merge size 8,
+ * interval size 8, CTA count 256, max registers 128) where they apply. */
+typedef struct {
+  uint32_t interval;       /* zero-block-skipping guard interval in IR instructions (Sec. 6); 0 = default 8; UINT32_MAX = no guards */
+  uint32_t max_regs;       /* NVRTC --maxrregcount; 0 = default 128 */
+  uint32_t group_size;     /* max regexes per group; 0 = auto */
+  uint32_t words_per_lane; /* K: 32-bit words per lane per window (window = 1024*K positions); 0 = auto */
+  uint32_t flags;          /* RX_F_* below */
+  uint32_t reserved[3];
+} rx_options;
+
+#define RX_F_NO_REBALANCE 1u /* disable Shift Rebalancing (Sec. 5) */
+#define RX_F_NO_GUARDS 2u    /* disable Zero Block Skipping (Sec. 6) */
+#define RX_F_NO_CACHE 4u     /* do not read/write the on-disk cubin cache */
+
+/* Compile n patterns (byte strings, not NUL-terminated).  On error returns
+ * the status and, if err != NULL, fills it.  *out owns everything. */
+rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, uint32_t n_patterns,
+                     const rx_options *opt /* nullable */, rx_program **out, rx_error *err /* nullable */);
+void rx_free(rx_program *p);
+
+uint32_t rx_num_regex(const rx_program *p);
+uint32_t rx_num_groups(const rx_program *p);
+/* Static halo in bytes a chunk needs before / after its committed range
+ * (DESIGN.md "Margins"): unbounded constructs are carried in the boundary
+ * state instead. */
+uint32_t rx_max_lookback(const rx_program *p);
+uint32_t rx_max_lookahead(const rx_program *p);
+/* Bytes of boundary state (MatchStar carries, forwarded loop tails). */
+size_t rx_boundary_bytes(const rx_program *p);
+/* The generated CUDA C source of the program (NUL-terminated, owned by p). */
+const char *rx_program_source(const rx_program *p);
+/* Human-readable IR / per-group geometry dump (owned by p). */
+const char *rx_program_info(const rx_program *p);
+
+typedef struct {
+  uint32_t regex;
+  uint32_t pad;
+  uint64_t pos;
+} rx_match_t;
+
+typedef struct {
+  uint64_t *d_counts;     /* required: u64[n_regex], OVERWRITTEN with the match counts */
+  uint64_t *d_digests;    /* nullable: u64[2*n_regex]: sum splitmix64(p), sum splitmix64(p^0x9E3779B97F4A7C15) */
+  uint32_t *d_bitstreams; /* nullable: u32[n_regex * pitch_words], LSB-first (bit p of word p/32); bits >= len are 0 */
+  uint64_t pitch_words;   /* >= ceil(len/32) when d_bitstreams != NULL */
+  uint32_t *d_status;     /* nullable: u32 device flags, bit0 = iteration cap hit (result not exact) */
+  uint32_t reserved[4];
+} rx_output;
+
+/* Match the whole input d_input[0..len).  Asynchronous on `stream`
+ * (a cudaStream_t; NULL = legacy default stream). */
+rx_status rx_match(const rx_program *p, const uint8_t *d_input, uint64_t len, void *stream, const rx_output *out);
+
+/* Chunked / multi-GPU form: commit positions [0, len) of a chunk whose bytes
+ * are readable at d_input[-halo_left .. len + halo_right).  Positions are
+ * reported as global_offset + i (digests, bitstreams stay chunk-relative).
+ * d_state_in: nullable device blob of rx_boundary_bytes() (NULL = the chunk
+ * starts the stream: zero state); d_state_out: nullable, receives the state
+ * at the chunk end.  Counts/digests are ACCUMULATED when `accumulate` != 0. */
+rx_status rx_match_chunk(const rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo_left,
+                         uint64_t halo_right, uint64_t global_offset, const void *d_state_in, void *d_state_out,
+                         int accumulate, void *stream, const rx_output *out);
+
+/* Correction for a chunk that was matched assuming d_state_assumed but whose
+ * true incoming state is d_state_true: re-runs windows from the chunk start
+ * until the two runs' states agree, adding (new - old) to counts/digests and
+ * rewriting bitstream words.  d_state_out receives the corrected end state
+ * (or is left untouched when the runs converge before the end). */
+rx_status rx_rematch_chunk(const rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo_left,
+                           uint64_t halo_right, uint64_t global_offset, const void *d_state_assumed,
+                           const void *d_state_true, void *d_state_out, void *stream, const rx_output *out);
+
+/* Last error message of this thread (static storage). */
+const char *rx_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* RX_H_ */

@@ -1,0 +1,227 @@
+"""B200-native interleaved bitstream regex matching (BitGen's hot path).
+
+Thin Python binding over the C ABI of ``include/rx.h`` (``librx.so``):
+argument marshalling only.  Every step of matching runs in the generated
+sm_100a kernels; there is no CPU fallback -- calls that compute raise
+``RxError`` when the library or a CUDA device is missing.
+
+PyTorch is used for device memory and streams only.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import threading
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_LIB_PATH = os.path.join(_HERE, "librx.so")
+_lock = threading.Lock()
+_lib = None
+
+RX_OK, RX_EPARSE, RX_EUNSUPPORTED, RX_ETOOBIG, RX_EJIT, RX_ECUDA, RX_EINVAL, RX_ENOMEM, RX_EOVERFLOW = range(9)
+RX_F_NO_REBALANCE, RX_F_NO_GUARDS, RX_F_NO_CACHE = 1, 2, 4
+
+EXPORTED = ["rx_compile", "rx_free", "rx_num_regex", "rx_num_groups", "rx_max_lookback", "rx_max_lookahead",
+            "rx_boundary_bytes", "rx_program_source", "rx_program_info", "rx_match", "rx_match_chunk",
+            "rx_rematch_chunk", "rx_last_error"]
+
+
+class RxError(RuntimeError):
+    def __init__(self, status, msg, index=None, offset=None):
+        super().__init__(f"rx status {status}: {msg}")
+        self.status, self.index, self.offset = status, index, offset
+
+
+class _Options(ctypes.Structure):
+    _fields_ = [("interval", ctypes.c_uint32), ("max_regs", ctypes.c_uint32), ("group_size", ctypes.c_uint32),
+                ("words_per_lane", ctypes.c_uint32), ("flags", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 3)]
+
+
+class _Error(ctypes.Structure):
+    _fields_ = [("pattern_index", ctypes.c_uint32), ("byte_offset", ctypes.c_uint32), ("msg", ctypes.c_char * 256)]
+
+
+class _Output(ctypes.Structure):
+    _fields_ = [("d_counts", ctypes.c_void_p), ("d_digests", ctypes.c_void_p), ("d_bitstreams", ctypes.c_void_p),
+                ("pitch_words", ctypes.c_uint64), ("d_status", ctypes.c_void_p), ("reserved", ctypes.c_uint32 * 4)]
+
+
+def lib_path() -> str:
+    return _LIB_PATH
+
+
+def load_library():
+    """Load librx.so (building it in-tree first if it is missing)."""
+    global _lib
+    with _lock:
+        if _lib is not None:
+            return _lib
+        if not os.path.exists(_LIB_PATH):
+            from . import build as _b
+            _b.build()
+        lib = ctypes.CDLL(_LIB_PATH)
+        vp, u32, u64, sz = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_size_t
+        lib.rx_compile.argtypes = [vp, vp, u32, ctypes.POINTER(_Options), ctypes.POINTER(vp), ctypes.POINTER(_Error)]
+        lib.rx_compile.restype = ctypes.c_int
+        lib.rx_free.argtypes = [vp]
+        for f in ("rx_num_regex", "rx_num_groups", "rx_max_lookback", "rx_max_lookahead"):
+            getattr(lib, f).argtypes = [vp]
+            getattr(lib, f).restype = u32
+        lib.rx_boundary_bytes.argtypes = [vp]
+        lib.rx_boundary_bytes.restype = sz
+        lib.rx_program_source.argtypes = [vp]
+        lib.rx_program_source.restype = ctypes.c_char_p
+        lib.rx_program_info.argtypes = [vp]
+        lib.rx_program_info.restype = ctypes.c_char_p
+        lib.rx_match.argtypes = [vp, vp, u64, vp, ctypes.POINTER(_Output)]
+        lib.rx_match.restype = ctypes.c_int
+        lib.rx_match_chunk.argtypes = [vp, vp, u64, u64, u64, u64, vp, vp, ctypes.c_int, vp, ctypes.POINTER(_Output)]
+        lib.rx_match_chunk.restype = ctypes.c_int
+        lib.rx_rematch_chunk.argtypes = [vp, vp, u64, u64, u64, u64, vp, vp, vp, vp, ctypes.POINTER(_Output)]
+        lib.rx_rematch_chunk.restype = ctypes.c_int
+        lib.rx_last_error.argtypes = []
+        lib.rx_last_error.restype = ctypes.c_char_p
+        _lib = lib
+        return lib
+
+
+def _check(status):
+    if status != RX_OK:
+        raise RxError(status, load_library().rx_last_error().decode("utf-8", "replace"))
+
+
+def _ptr(t):
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+def _stream_handle(stream):
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+class Program:
+    """A compiled pattern set (rx_compile)."""
+
+    def __init__(self, patterns, interval=None, max_regs=None, group_size=None, words_per_lane=None, flags=0):
+        lib = load_library()
+        pats = [p.encode("latin-1") if isinstance(p, str) else bytes(p) for p in patterns]
+        self.patterns = pats
+        n = len(pats)
+        bufs = [ctypes.create_string_buffer(p, len(p) + 1) for p in pats]
+        arr = (ctypes.c_void_p * max(n, 1))(*[ctypes.cast(b, ctypes.c_void_p) for b in bufs])
+        lens = (ctypes.c_size_t * max(n, 1))(*[len(p) for p in pats])
+        opt = _Options()
+        opt.interval = 0 if interval is None else (0xFFFFFFFF if interval <= 0 else int(interval))
+        opt.max_regs = int(max_regs or 0)
+        opt.group_size = int(group_size or 0)
+        opt.words_per_lane = int(words_per_lane or 0)
+        opt.flags = int(flags)
+        err = _Error()
+        h = ctypes.c_void_p()
+        st = lib.rx_compile(arr, lens, n, ctypes.byref(opt), ctypes.byref(h), ctypes.byref(err))
+        if st != RX_OK:
+            raise RxError(st, lib.rx_last_error().decode("utf-8", "replace"), err.pattern_index, err.byte_offset)
+        self._h = h
+        self._lib = lib
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h is not None and h.value:
+            self._lib.rx_free(h)
+            self._h = None
+
+    # --- properties ---------------------------------------------------------
+    @property
+    def n_regex(self) -> int:
+        return int(self._lib.rx_num_regex(self._h))
+
+    @property
+    def n_groups(self) -> int:
+        return int(self._lib.rx_num_groups(self._h))
+
+    @property
+    def lookback(self) -> int:
+        return int(self._lib.rx_max_lookback(self._h))
+
+    @property
+    def lookahead(self) -> int:
+        return int(self._lib.rx_max_lookahead(self._h))
+
+    @property
+    def boundary_bytes(self) -> int:
+        return int(self._lib.rx_boundary_bytes(self._h))
+
+    @property
+    def source(self) -> str:
+        return self._lib.rx_program_source(self._h).decode()
+
+    @property
+    def info(self) -> str:
+        return self._lib.rx_program_info(self._h).decode()
+
+    # --- matching -----------------------------------------------------------
+    def alloc_outputs(self, length, device=None, dense=False, digests=True):
+        import torch
+        device = device or torch.device("cuda", torch.cuda.current_device())
+        n = self.n_regex
+        out = {"counts": torch.zeros(max(n, 1), dtype=torch.int64, device=device)[:n],
+               "digests": torch.zeros((max(n, 1), 2), dtype=torch.int64, device=device)[:n] if digests else None,
+               "status": torch.zeros(1, dtype=torch.int32, device=device)}
+        if dense:
+            pitch = max((int(length) + 31) // 32, 1)
+            out["dense"] = torch.zeros((max(n, 1), pitch), dtype=torch.int32, device=device)[:n]
+            out["pitch"] = pitch
+        else:
+            out["dense"], out["pitch"] = None, 0
+        return out
+
+    def _out_struct(self, o):
+        s = _Output()
+        s.d_counts = o["counts"].data_ptr()
+        s.d_digests = o["digests"].data_ptr() if o.get("digests") is not None else None
+        s.d_bitstreams = o["dense"].data_ptr() if o.get("dense") is not None else None
+        s.pitch_words = int(o.get("pitch") or 0)
+        s.d_status = o["status"].data_ptr() if o.get("status") is not None else None
+        return s
+
+    def match(self, data, out=None, dense=False, digests=True, stream=None):
+        """Match a CUDA uint8 tensor; returns dict(counts=int64[n] (u64 bits),
+        digests=int64[n,2], dense=int32[n, pitch] LSB-first, status)."""
+        if out is None:
+            out = self.alloc_outputs(data.numel(), data.device, dense=dense, digests=digests)
+        s = self._out_struct(out)
+        _check(self._lib.rx_match(self._h, _ptr(data), int(data.numel()), _stream_handle(stream), ctypes.byref(s)))
+        return out
+
+    def match_chunk(self, data, length, halo_left, halo_right, global_offset, state_in=None, state_out=None,
+                    out=None, accumulate=False, dense=False, digests=True, stream=None):
+        """`data` is a CUDA uint8 tensor holding [halo_left | chunk(length) | halo_right]."""
+        if out is None:
+            out = self.alloc_outputs(length, data.device, dense=dense, digests=digests)
+        s = self._out_struct(out)
+        base = data.data_ptr() + int(halo_left)
+        _check(self._lib.rx_match_chunk(self._h, ctypes.c_void_p(base), int(length), int(halo_left), int(halo_right),
+                                        int(global_offset), _ptr(state_in), _ptr(state_out), int(bool(accumulate)),
+                                        _stream_handle(stream), ctypes.byref(s)))
+        return out
+
+    def rematch_chunk(self, data, length, halo_left, halo_right, global_offset, state_assumed, state_true,
+                      state_out, out, stream=None):
+        s = self._out_struct(out)
+        base = data.data_ptr() + int(halo_left)
+        _check(self._lib.rx_rematch_chunk(self._h, ctypes.c_void_p(base), int(length), int(halo_left),
+                                          int(halo_right), int(global_offset), _ptr(state_assumed),
+                                          _ptr(state_true), _ptr(state_out), _stream_handle(stream),
+                                          ctypes.byref(s)))
+        return out
+
+    def new_state(self, device=None):
+        import torch
+        device = device or torch.device("cuda", torch.cuda.current_device())
+        return torch.zeros(max(self.boundary_bytes // 4, 1), dtype=torch.int32, device=device)
+
+
+def compile(patterns, **kw) -> Program:  # noqa: A001 (mirrors rx_compile)
+    return Program(patterns, **kw)

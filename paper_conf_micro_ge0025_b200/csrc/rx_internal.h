@@ -1,0 +1,135 @@
+// rx_internal.h -- host compiler internals: AST, bitstream IR, groups.
+//
+// PAPER.md references (P:Lnnn): grammar P:L67-69 (Listing 1 lost);
+// lowering rules Fig. 2 and Listing 3; bitstream
+// program grammar P:L118 (Listing 2 lost).
+#pragma once
+#include <cstdint>
+#include <memory>
+#include <string>
+#include <vector>
+
+namespace rx {
+
+// 256-bit byte set.
+struct ByteSet {
+  uint64_t w[4] = {0, 0, 0, 0};
+  void set(int c) { w[c >> 6] |= 1ull << (c & 63); }
+  bool has(int c) const { return (w[c >> 6] >> (c & 63)) & 1; }
+  void range(int a, int b) { for (int c = a; c <= b; ++c) set(c); }
+  void invert() { for (auto &x : w) x = ~x; }
+  void merge(const ByteSet &o) { for (int i = 0; i < 4; ++i) w[i] |= o.w[i]; }
+  bool empty() const { return !(w[0] | w[1] | w[2] | w[3]); }
+  bool full() const { return !~(w[0] & w[1] & w[2] & w[3]); }
+  int count() const { int n = 0; for (auto x : w) n += __builtin_popcountll(x); return n; }
+  bool operator==(const ByteSet &o) const { return w[0] == o.w[0] && w[1] == o.w[1] && w[2] == o.w[2] && w[3] == o.w[3]; }
+};
+
+// ----------------------------------------------------------------------------
+// AST (the compiler's own parser; the oracle has a separate one)
+// ----------------------------------------------------------------------------
+enum class AK : uint8_t { Empty, Set, Cat, Alt, Rep };
+struct Ast {
+  AK kind = AK::Empty;
+  ByteSet set;                       // Set
+  std::vector<std::unique_ptr<Ast>> kids;  // Cat / Alt: items; Rep: kids[0]
+  int lo = 0, hi = 0;                // Rep: hi < 0 = unbounded
+};
+using AstP = std::unique_ptr<Ast>;
+
+struct ParseError {
+  int code;  // rx_status: 1 parse, 2 unsupported, 3 too big
+  size_t at;
+  std::string msg;
+};
+
+// Returns nullptr and fills err on failure.
+AstP parse_regex(const std::string &pat, ParseError &err);
+bool ast_nullable(const Ast &a);
+size_t ast_expanded_size(const Ast &a);  // #Set leaves after R{n,m} expansion (for caps)
+
+// ----------------------------------------------------------------------------
+// Bitstream IR (per regex).  Streams are indexed by input position p (bit p of
+// word p/32, LSB-first; SURVEY App.A-1).  Paper's "S >> k" (advance) = Adv.
+// ----------------------------------------------------------------------------
+enum class Op : uint8_t {
+  Zero,    // all-zero stream
+  Ones,    // all-ones stream incl. positions < 0 (the unanchored start marker, DESIGN "start")
+  CC,      // character class from the basis streams (Fig. 2a)
+  And, Or, Xor, AndNot,  // AndNot(a,b) = a & ~b
+  Adv,     // out[p] = in[p-k]  (paper ">> k", Fig. 2b); inside loop bodies: forwarded site
+  Look,    // out[p] = in[p+k]  (paper "<< k", produced by Shift Rebalancing)
+  MStar,   // ends of X C*: ((((X + C) ^ C) | X) & C), X subset C (MatchStar, Parabix [24])
+  Loop,    // while-fixpoint of Fig. 2e / Listing 3: acc = lfp(seeds U body(acc))
+  Fr,      // the frontier placeholder inside a Loop body
+  Guard,   // zero-block-skipping region (Sec. 6): value = region result, or 0 if any(cond)==0
+};
+
+struct Node {
+  Op op = Op::Zero;
+  int a = -1, b = -1;  // operands (node ids); Guard: a = condition; Loop: a = seeds
+  int k = 0;           // Adv / Look distance
+  int cc = -1;         // CC: index into Program::sets
+  int sub = -1;        // Loop / Guard: body block id
+  int res = -1;        // Loop: body result E(R, Fr); Guard: region result
+  int fr = -1;         // Loop: its Fr node
+  int loop = -1;       // innermost enclosing Loop node (-1: top level)
+  // analysis
+  int lb = 0, rb = 0;  // invalid bits at the window's left / right edge (margins, DESIGN "Margins")
+  int aw = 0;          // stateful: injection word (MStar, forwarded Adv, Loop)
+  int slot = -1;       // stateful: state slot (MStar carry, forwarded Adv tail)
+  int depth = 0;       // longest op path from inputs (Shift Rebalancing)
+};
+
+struct Block {
+  std::vector<int> nodes;  // emission order
+};
+
+struct RegexIR {
+  std::vector<Node> nodes;
+  std::vector<Block> blocks;  // blocks[0] = top level
+  std::vector<ByteSet> sets;
+  int out = -1;               // result node (top level)
+  int nslots = 0;
+  int lb = 0, rb = 0;         // margins of the output (bits)
+  int rb_state = 0;           // max rb over inputs of stateful sites (bits)
+  size_t n_instr = 0;         // instruction count (for grouping / guards)
+  int n_loops = 0, n_mstar = 0, n_adv = 0, n_guards = 0;
+};
+
+struct LowerOptions {
+  int interval = 8;       // guard interval (instructions), <= 0: no guards
+  bool rebalance = true;
+};
+
+// Lower one parsed regex to IR (non-empty, unanchored match ends).
+void lower_regex(const Ast &ast, const LowerOptions &opt, RegexIR &ir);
+// Compute margins, injection words and state slots.  Returns false if a
+// construct is not representable (message in why).
+bool analyze_regex(RegexIR &ir, std::string &why);
+std::string dump_ir(const RegexIR &ir);
+
+// ----------------------------------------------------------------------------
+// Groups and program geometry
+// ----------------------------------------------------------------------------
+struct Group {
+  std::vector<int> regexes;  // global regex ids
+  int K = 1;                 // words per lane per window
+  int Lw = 0, Rw = 0, Bw = 0;  // window: left halo words, right halo words, committed words (32K = Lw+Bw+Rw)
+  int nslots = 0;
+  std::vector<int> slot_base;  // per member regex
+  double cost = 0;
+};
+
+struct CompiledSet {
+  std::vector<RegexIR> irs;
+  std::vector<Group> groups;
+  std::string source;  // generated CUDA C
+  std::string info;
+};
+
+// CUDA C source of groups [g_begin, g_end) as one module (slot base sbase0).
+std::string emit_program_source_range(CompiledSet &cs, int g_begin, int g_end, uint32_t sbase0);
+bool plan_groups(CompiledSet &cs, int group_size, int force_K, std::string &why);
+
+}  // namespace rx

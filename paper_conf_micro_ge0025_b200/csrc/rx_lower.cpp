@@ -1,0 +1,513 @@
+// rx_lower.cpp -- lowering regexes to the bitstream IR, margin analysis,
+// Shift Rebalancing, zero-block guards, grouping.
+//
+// Lowering follows PAPER.md Fig. 2 in the end-position
+// convention of P:L120 ("a 1 at position i indicates a successful match
+// ending at that position"):
+//   E(CC, M)        = Adv(M, 1) & CC                       Fig. 2b
+//   E(R1|R2, M)     = E(R1, M) | E(R2, M)                  Fig. 2c
+//   E(R{n,m}, M)    = unrolled concatenation, OR of the n..m chains  Fig. 2d
+//   E(R+, M)        = while-fixpoint with frontier/acc     Fig. 2e, Listing 3
+//   E(CC+, M)       = MatchStar (one add with carry)       Parabix [24]
+// M = Ones is the unanchored start ("R1 is used as a prefix to determine the
+// starting positions"; every position may start).  Only non-empty
+// matches are produced (reading c1): R? and R* contribute their non-empty
+// part; concatenation tracks P (prefix may be empty) and N (non-empty).
+#include <algorithm>
+#include <cassert>
+#include <cstring>
+#include <functional>
+#include <map>
+#include <sstream>
+#include <tuple>
+
+#include "rx_internal.h"
+
+namespace rx {
+namespace {
+
+struct Key {
+  Op op;
+  int a, b, k, cc;
+  bool operator<(const Key &o) const {
+    return std::tie(op, a, b, k, cc) < std::tie(o.op, o.a, o.b, o.k, o.cc);
+  }
+};
+
+struct Item {
+  const Ast *ast;
+  enum Mode { Once, Opt, Plus } mode;
+};
+
+struct Lowerer {
+  RegexIR &ir;
+  LowerOptions opt;
+  std::vector<int> blk;                     // block stack
+  std::vector<int> loops;                   // enclosing loop nodes
+  std::vector<std::map<Key, int>> cse;      // scoped hash-consing
+  std::map<std::vector<uint64_t>, int> set_ix;
+  int zero = -1, ones = -1;
+  size_t since_guard = 0;
+
+  Lowerer(RegexIR &r, const LowerOptions &o) : ir(r), opt(o) {}
+
+  int cur_loop() const { return loops.empty() ? -1 : loops.back(); }
+
+  int raw(Node n) {
+    n.loop = cur_loop();
+    ir.nodes.push_back(n);
+    int id = (int)ir.nodes.size() - 1;
+    ir.blocks[blk.back()].nodes.push_back(id);
+    ir.n_instr++;
+    since_guard++;
+    return id;
+  }
+
+  int mk(Op op, int a = -1, int b = -1, int k = 0, int cc = -1) {
+    if ((op == Op::And || op == Op::Or || op == Op::Xor) && a > b) std::swap(a, b);
+    Key key{op, a, b, k, cc};
+    for (auto it = cse.rbegin(); it != cse.rend(); ++it) {
+      auto f = it->find(key);
+      if (f != it->end()) return f->second;
+    }
+    Node n;
+    n.op = op;
+    n.a = a;
+    n.b = b;
+    n.k = k;
+    n.cc = cc;
+    int id = raw(n);
+    cse.back()[key] = id;
+    return id;
+  }
+
+  int push_block() {
+    ir.blocks.emplace_back();
+    int id = (int)ir.blocks.size() - 1;
+    blk.push_back(id);
+    cse.emplace_back();
+    return id;
+  }
+  void pop_block() {
+    blk.pop_back();
+    cse.pop_back();
+  }
+
+  bool is(int v, Op op) const { return ir.nodes[v].op == op; }
+
+  // --- constant-folding constructors -------------------------------------
+  int Zero() { return zero; }
+  int AND(int a, int b) {
+    if (is(a, Op::Zero) || is(b, Op::Zero)) return zero;
+    if (is(a, Op::Ones)) return b;
+    if (is(b, Op::Ones)) return a;
+    if (a == b) return a;
+    return mk(Op::And, a, b);
+  }
+  int OR(int a, int b) {
+    if (is(a, Op::Zero)) return b;
+    if (is(b, Op::Zero)) return a;
+    if (is(a, Op::Ones) || is(b, Op::Ones)) return ones;
+    if (a == b) return a;
+    return mk(Op::Or, a, b);
+  }
+  int ADV1(int m) {
+    if (is(m, Op::Zero)) return zero;
+    if (is(m, Op::Ones)) return ones;  // the virtual start at position -1 (P:L116 prefix)
+    return mk(Op::Adv, m, -1, 1);
+  }
+  int CC(const ByteSet &s) {
+    if (s.empty()) return zero;
+    std::vector<uint64_t> key(s.w, s.w + 4);
+    int ix;
+    auto f = set_ix.find(key);
+    if (f == set_ix.end()) {
+      ix = (int)ir.sets.size();
+      ir.sets.push_back(s);
+      set_ix[key] = ix;
+    } else {
+      ix = f->second;
+    }
+    return mk(Op::CC, -1, -1, 0, ix);
+  }
+
+  // --- E(R, M) -------------------------------------------------------------
+  static const Ast *single_set(const Ast &a, ByteSet &out) {
+    // A sub-expression that matches exactly one byte from a set: Set, or
+    // Alt of single sets, or Rep{1,1} of one.
+    if (a.kind == AK::Set) { out = a.set; return &a; }
+    if (a.kind == AK::Alt) {
+      ByteSet u;
+      for (auto &k : a.kids) {
+        ByteSet s;
+        if (!single_set(*k, s)) return nullptr;
+        u.merge(s);
+      }
+      out = u;
+      return &a;
+    }
+    if (a.kind == AK::Rep && a.lo == 1 && a.hi == 1) return single_set(*a.kids[0], out);
+    if (a.kind == AK::Cat && a.kids.size() == 1) return single_set(*a.kids[0], out);
+    return nullptr;
+  }
+
+  int E(const Ast &r, int M) {
+    if (is(M, Op::Zero)) return zero;
+    switch (r.kind) {
+      case AK::Empty: return zero;
+      case AK::Set: return AND(ADV1(M), CC(r.set));
+      case AK::Alt: {
+        int acc = zero;
+        for (auto &k : r.kids) acc = OR(acc, E(*k, M));
+        return acc;
+      }
+      case AK::Cat: {
+        std::vector<Item> items;
+        for (auto &k : r.kids) items.push_back({k.get(), Item::Once});
+        return E_cat(items, 0, M, zero);
+      }
+      case AK::Rep: {
+        const Ast &kid = *r.kids[0];
+        if (r.hi == 0) return zero;
+        std::vector<Item> items;
+        if (r.hi < 0) {
+          for (int i = 0; i + 1 < r.lo; ++i) items.push_back({&kid, Item::Once});
+          items.push_back({&kid, Item::Plus});
+        } else {
+          for (int i = 0; i < r.lo; ++i) items.push_back({&kid, Item::Once});
+          for (int i = r.lo; i < r.hi; ++i) items.push_back({&kid, Item::Opt});
+        }
+        return E_cat(items, 0, M, zero);
+      }
+    }
+    return zero;
+  }
+
+  int E_item(const Item &it, int P) {
+    switch (it.mode) {
+      case Item::Once:
+      case Item::Opt: return E(*it.ast, P);
+      case Item::Plus: return E_plus(*it.ast, P);
+    }
+    return zero;
+  }
+  bool item_nullable(const Item &it) {
+    return it.mode == Item::Opt || ast_nullable(*it.ast);
+  }
+
+  // Concatenation items[j..] after a prefix whose (possibly empty) end
+  // markers are P and whose non-empty end markers are N.
+  int E_cat(const std::vector<Item> &items, size_t j, int P, int N) {
+    for (; j < items.size(); ++j) {
+      // Zero-block-skipping guard (Sec. 6): P is a zero-path
+      // head -- if P is all-zero in a window, everything downstream in this
+      // concatenation (and N, a subset of P) is zero.  First guard after the
+      // first shift+AND, then every `interval` instructions.
+      if (opt.interval > 0 && loops.empty() && j > 0 && !is(P, Op::Ones) && !is(P, Op::Zero) &&
+          since_guard >= (size_t)opt.interval && ir.nodes[P].op != Op::CC) {
+        Node g;
+        g.op = Op::Guard;
+        g.a = P;
+        int gid = raw(g);
+        ir.n_guards++;
+        int sb = push_block();
+        since_guard = 0;
+        int res = E_cat(items, j, P, N);
+        pop_block();
+        ir.nodes[gid].sub = sb;
+        ir.nodes[gid].res = res;
+        if (is(res, Op::Zero)) return zero;
+        return gid;
+      }
+      const Item &it = items[j];
+      int e = E_item(it, P);
+      if (item_nullable(it)) {
+        int nP = OR(e, P);
+        N = OR(e, N);
+        P = nP;
+      } else {
+        P = e;
+        N = e;
+      }
+      if (j == 0 && ir.n_guards == 0) since_guard = std::max<size_t>(since_guard, 0);
+      if (is(P, Op::Zero)) return zero;
+    }
+    return N;
+  }
+
+  // E(R+, M): non-empty repetitions of R after prefix ends M.
+  int E_plus(const Ast &r, int M) {
+    ByteSet s;
+    if (single_set(r, s)) {
+      if (s.empty()) return zero;
+      int C = CC(s);
+      if (is(M, Op::Ones)) return C;  // every C position ends a one-byte match
+      int X = AND(ADV1(M), C);
+      if (is(X, Op::Zero)) return zero;
+      Node n;
+      n.op = Op::MStar;
+      n.a = X;
+      n.b = C;
+      ir.n_mstar++;
+      return raw(n);  // stateful: never hash-consed
+    }
+    // General body: while-fixpoint (Fig. 2e, Listing 3).  The frontier
+    // starts at the prefix ends M itself, so the body E(r, .) is lowered
+    // once: acc = U_i E(r, fr_i), fr_0 = M, fr_{i+1} = E(r, fr_i) & ~acc.
+    // (At the unanchored start M = Ones, seed the loop with E(r, Ones) --
+    // the virtual start position has no bit in the window.)
+    int seeds = M;
+    if (is(M, Op::Ones)) {
+      int e = E(r, M);
+      if (is(e, Op::Zero)) return zero;
+      Node L0;
+      L0.op = Op::Loop;
+      L0.a = e;
+      L0.k = 1;  // k=1: seeds are ends of r already (acc starts with them)
+      int lid0 = raw(L0);
+      ir.n_loops++;
+      lower_body(lid0, r);
+      return lid0;
+    }
+    Node L;
+    L.op = Op::Loop;
+    L.a = seeds;
+    L.k = 0;  // k=0: seeds are prefix ends (frontier only, not in acc)
+    int lid = raw(L);
+    ir.n_loops++;
+    lower_body(lid, r);
+    return lid;
+  }
+
+  void lower_body(int lid, const Ast &r) {
+    int sb = push_block();
+    loops.push_back(lid);
+    Node f;
+    f.op = Op::Fr;
+    int fr = raw(f);
+    int res = E(r, fr);
+    loops.pop_back();
+    pop_block();
+    ir.nodes[lid].sub = sb;
+    ir.nodes[lid].fr = fr;
+    ir.nodes[lid].res = res;
+  }
+};
+
+}  // namespace
+
+void lower_regex(const Ast &ast, const LowerOptions &opt, RegexIR &ir) {
+  ir = RegexIR();
+  ir.blocks.emplace_back();
+  Lowerer L(ir, opt);
+  L.blk.push_back(0);
+  L.cse.emplace_back();
+  Node z;
+  z.op = Op::Zero;
+  L.zero = L.raw(z);
+  Node o;
+  o.op = Op::Ones;
+  L.ones = L.raw(o);
+  L.since_guard = 0;
+  ir.n_instr = 0;
+  ir.out = L.E(ast, L.ones);
+  if (ir.out == L.ones) {
+    // a regex matching every position with a one-byte match of [\x00-\xff]
+    // cannot lower to Ones (Ones is 1 at padding too); E never returns Ones
+    // for a non-empty R, keep the guard anyway.
+    ir.out = L.CC([] { ByteSet s; s.range(0, 255); return s; }());
+  }
+}
+
+// ----------------------------------------------------------------------------
+// Margins: a window frame computes words [0, 32K); a
+// value v is exact at bit positions [lb(v), 32K*32 - rb(v)).  Static shifts
+// grow the margins (the paper's overlap distance, generalised to
+// per-side margins, SURVEY App.A-8); unbounded constructs (MatchStar, while
+// loops) are exact from their injection word aw on, with their cross-window
+// dependency carried as state.
+// ----------------------------------------------------------------------------
+static void mark_loop_sites(RegexIR &ir, int block, int aw, int &slot) {
+  for (int id : ir.blocks[block].nodes) {
+    Node &n = ir.nodes[id];
+    switch (n.op) {
+      case Op::Adv:
+        if (n.k > 32) n.k = 32;  // (bodies only produce Adv 1)
+        n.aw = aw;
+        n.slot = slot++;
+        break;
+      case Op::MStar:
+        n.aw = aw;
+        n.slot = slot++;
+        break;
+      case Op::Loop:
+        n.aw = aw;
+        mark_loop_sites(ir, n.sub, aw, slot);
+        break;
+      case Op::Guard:
+        mark_loop_sites(ir, n.sub, aw, slot);
+        break;
+      default:
+        break;
+    }
+  }
+}
+
+static void margins_block(RegexIR &ir, int block, int &slot) {
+  for (int id : ir.blocks[block].nodes) {
+    Node &n = ir.nodes[id];
+    auto lb = [&](int x) { return ir.nodes[x].lb; };
+    auto rb = [&](int x) { return ir.nodes[x].rb; };
+    auto dp = [&](int x) { return ir.nodes[x].depth; };
+    switch (n.op) {
+      case Op::Zero: case Op::Ones: case Op::CC: case Op::Fr:
+        n.lb = n.rb = 0;
+        n.depth = 0;
+        break;
+      case Op::And: case Op::Or: case Op::Xor: case Op::AndNot:
+        n.lb = std::max(lb(n.a), lb(n.b));
+        n.rb = std::max(rb(n.a), rb(n.b));
+        n.depth = std::max(dp(n.a), dp(n.b)) + 1;
+        break;
+      case Op::Adv:
+        n.lb = lb(n.a) + n.k;
+        n.rb = std::max(rb(n.a) - n.k, 0);
+        n.depth = dp(n.a) + 1;
+        break;
+      case Op::Look:
+        n.lb = std::max(lb(n.a) - n.k, 0);
+        n.rb = rb(n.a) + n.k;
+        n.depth = dp(n.a) + 1;
+        break;
+      case Op::MStar: {
+        int l = std::max(lb(n.a), lb(n.b));
+        n.aw = (l + 31) / 32;
+        n.slot = slot++;
+        n.lb = 32 * n.aw;
+        n.rb = std::max(rb(n.a), rb(n.b));
+        n.depth = std::max(dp(n.a), dp(n.b)) + 4;
+        ir.rb_state = std::max(ir.rb_state, n.rb);
+        break;
+      }
+      case Op::Loop: {
+        // body invariants are CCs (lb 0); seeds carry the static part
+        n.aw = (lb(n.a) + 31) / 32 + 1;
+        mark_loop_sites(ir, n.sub, n.aw, slot);
+        n.lb = 32 * n.aw;
+        n.rb = rb(n.a);
+        n.depth = dp(n.a) + 8;
+        ir.rb_state = std::max(ir.rb_state, n.rb);
+        break;
+      }
+      case Op::Guard: {
+        margins_block(ir, n.sub, slot);
+        n.lb = lb(n.res);
+        n.rb = rb(n.res);
+        n.depth = dp(n.res);
+        break;
+      }
+    }
+  }
+}
+
+bool analyze_regex(RegexIR &ir, std::string &why) {
+  int slot = 0;
+  margins_block(ir, 0, slot);
+  ir.nslots = slot;
+  ir.lb = ir.nodes[ir.out].lb;
+  ir.rb = ir.nodes[ir.out].rb;
+  (void)why;
+  return true;
+}
+
+std::string dump_ir(const RegexIR &ir) {
+  static const char *names[] = {"zero", "ones", "cc", "and", "or", "xor", "andn", "adv", "look",
+                                "mstar", "loop", "fr", "guard"};
+  std::ostringstream os;
+  std::function<void(int, int)> blk = [&](int b, int ind) {
+    for (int id : ir.blocks[b].nodes) {
+      const Node &n = ir.nodes[id];
+      os << std::string(ind, ' ') << "v" << id << " = " << names[(int)n.op];
+      if (n.a >= 0) os << " v" << n.a;
+      if (n.b >= 0) os << " v" << n.b;
+      if (n.op == Op::Adv || n.op == Op::Look) os << " k=" << n.k;
+      if (n.op == Op::CC) os << " set#" << n.cc;
+      os << "   [lb=" << n.lb << " rb=" << n.rb;
+      if (n.slot >= 0) os << " slot=" << n.slot << " aw=" << n.aw;
+      if (n.loop >= 0) os << " in-loop v" << n.loop;
+      os << "]\n";
+      if (n.op == Op::Loop || n.op == Op::Guard) {
+        blk(n.sub, ind + 2);
+        os << std::string(ind + 2, ' ') << "-> v" << n.res << "\n";
+      }
+    }
+  };
+  blk(0, 0);
+  os << "out = v" << ir.out << " lb=" << ir.lb << " rb=" << ir.rb << " slots=" << ir.nslots << "\n";
+  return os.str();
+}
+
+// ----------------------------------------------------------------------------
+// Grouping ("Regexes are partitioned into groups with similar
+// total character length, each assigned to one CTA").  Here a group is the
+// program one warp runs over its windows; regexes are sorted by static span
+// so that a group's window geometry (K, halos) fits all members, then packed
+// greedily by instruction count.
+// ----------------------------------------------------------------------------
+bool plan_groups(CompiledSet &cs, int group_size, int force_K, std::string &why) {
+  int n = (int)cs.irs.size();
+  std::vector<int> order(n);
+  for (int i = 0; i < n; ++i) order[i] = i;
+  auto span = [&](int r) { return (cs.irs[r].lb + 31) / 32 + (std::max(cs.irs[r].rb, cs.irs[r].rb_state) + 31) / 32; };
+  std::stable_sort(order.begin(), order.end(), [&](int a, int b) { return span(a) < span(b); });
+  size_t total_instr = 0;
+  for (auto &r : cs.irs) total_instr += r.n_instr;
+  if (group_size <= 0) {
+    // aim for <= ~64 regexes and a bounded code size per group
+    group_size = 16;
+  }
+  const size_t max_instr = 600;
+  cs.groups.clear();
+  Group g;
+  size_t gi = 0;
+  for (int r : order) {
+    if (!g.regexes.empty() && ((int)g.regexes.size() >= group_size || gi + cs.irs[r].n_instr > max_instr)) {
+      cs.groups.push_back(g);
+      g = Group();
+      gi = 0;
+    }
+    g.regexes.push_back(r);
+    gi += cs.irs[r].n_instr;
+    g.cost += (double)cs.irs[r].n_instr;
+  }
+  if (!g.regexes.empty() || cs.groups.empty()) cs.groups.push_back(g);
+  for (auto &gr : cs.groups) {
+    int L = 0, R = 0;
+    gr.nslots = 0;
+    gr.slot_base.clear();
+    for (int r : gr.regexes) {
+      const RegexIR &ir = cs.irs[r];
+      L = std::max(L, (ir.lb + 31) / 32);
+      R = std::max(R, (std::max(ir.rb, ir.rb_state) + 31) / 32);
+      gr.slot_base.push_back(gr.nslots);
+      gr.nslots += ir.nslots;
+    }
+    int K = force_K;
+    if (K <= 0) {
+      K = 8;
+      for (int k : {1, 2, 4, 8})
+        if (4 * (L + R) <= 32 * k) { K = k; break; }
+    }
+    if (L + R >= 32 * K) {
+      why = "static span of a group exceeds the window (" + std::to_string(L + R) + " words)";
+      return false;
+    }
+    gr.K = K;
+    gr.Lw = L;
+    gr.Rw = R;
+    gr.Bw = 32 * K - L - R;
+  }
+  return true;
+}
+
+}  // namespace rx

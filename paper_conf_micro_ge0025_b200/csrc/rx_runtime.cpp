@@ -1,0 +1,534 @@
+// rx_runtime.cpp -- the C ABI (include/rx.h): compile (parse -> IR -> groups
+// -> CUDA C -> NVRTC sm_100a cubin, "compiled at runtime
+// using NVRTC"), lazy module load, and the launches of the fused kernel.
+//
+// There is no CPU execution path: rx_match / rx_match_chunk / rx_rematch_chunk
+// launch the generated sm_100a kernels or fail with RX_ECUDA.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <nvrtc.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <fstream>
+#include <mutex>
+#include <sstream>
+#include <string>
+#include <sys/stat.h>
+#include <thread>
+#include <unistd.h>
+#include <vector>
+
+#include "../../include/rx.h"
+#include "rx_internal.h"
+
+namespace {
+
+thread_local std::string g_last_error;
+
+rx_status fail(rx_status s, const std::string &m) {
+  g_last_error = m;
+  return s;
+}
+
+// ---------------------------------------------------------------------------
+// driver entry points (no link-time libcuda dependency: the .so loads on a
+// GPU-less host; module load happens at the first match)
+// ---------------------------------------------------------------------------
+struct Drv {
+  CUresult (*ModuleLoadData)(CUmodule *, const void *) = nullptr;
+  CUresult (*ModuleGetFunction)(CUfunction *, CUmodule, const char *) = nullptr;
+  CUresult (*LaunchKernel)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
+                           CUstream, void **, void **) = nullptr;
+  CUresult (*FuncSetAttribute)(CUfunction, CUfunction_attribute, int) = nullptr;
+  CUresult (*ModuleUnload)(CUmodule) = nullptr;
+  bool ok = false;
+  std::string why;
+};
+
+Drv &drv() {
+  static Drv d;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    auto get = [](const char *name, void **fn) -> bool {
+      cudaDriverEntryPointQueryResult q;
+      cudaError_t e = cudaGetDriverEntryPointByVersion(name, fn, 12000, cudaEnableDefault, &q);
+      return e == cudaSuccess && q == cudaDriverEntryPointSuccess && *fn;
+    };
+    bool ok = get("cuModuleLoadData", (void **)&d.ModuleLoadData) &&
+              get("cuModuleGetFunction", (void **)&d.ModuleGetFunction) &&
+              get("cuLaunchKernel", (void **)&d.LaunchKernel) &&
+              get("cuFuncSetAttribute", (void **)&d.FuncSetAttribute) &&
+              get("cuModuleUnload", (void **)&d.ModuleUnload);
+    d.ok = ok;
+    if (!ok) d.why = "CUDA driver entry points unavailable (no GPU / driver?)";
+  });
+  return d;
+}
+
+// ---------------------------------------------------------------------------
+// cubin cache
+// ---------------------------------------------------------------------------
+uint64_t fnv1a(const std::string &s, uint64_t h = 1469598103934665603ull) {
+  for (unsigned char c : s) {
+    h ^= c;
+    h *= 1099511628211ull;
+  }
+  return h;
+}
+
+std::string cache_dir() {
+  const char *e = getenv("RX_CACHE_DIR");
+  std::string d;
+  if (e && *e) d = e;
+  else {
+    const char *h = getenv("HOME");
+    d = std::string(h ? h : "/tmp") + "/.cache/bitrx";
+  }
+  return d;
+}
+
+void mkdirs(const std::string &d) {
+  std::string cur;
+  for (size_t i = 0; i < d.size(); ++i) {
+    cur += d[i];
+    if (d[i] == '/' && i > 0) mkdir(cur.c_str(), 0755);
+  }
+  mkdir(d.c_str(), 0755);
+}
+
+bool read_file(const std::string &path, std::string &out) {
+  std::ifstream f(path, std::ios::binary);
+  if (!f) return false;
+  std::ostringstream ss;
+  ss << f.rdbuf();
+  out = ss.str();
+  return !out.empty();
+}
+
+void write_file_atomic(const std::string &path, const std::string &data) {
+  std::string tmp = path + ".tmp" + std::to_string(getpid()) + "_" +
+                    std::to_string(std::hash<std::thread::id>()(std::this_thread::get_id()));
+  {
+    std::ofstream f(tmp, std::ios::binary);
+    if (!f) return;
+    f.write(data.data(), (std::streamsize)data.size());
+  }
+  rename(tmp.c_str(), path.c_str());
+}
+
+bool nvrtc_compile(const std::string &src, int max_regs, bool use_cache, std::string &cubin, std::string &log) {
+  int maj = 0, mnr = 0;
+  nvrtcVersion(&maj, &mnr);
+  std::vector<std::string> opts = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo", "-default-device",
+                                   "--maxrregcount=" + std::to_string(max_regs), "-DNDEBUG"};
+  std::string key_src = src;
+  for (auto &o : opts) key_src += "\n//" + o;
+  key_src += "\n//nvrtc " + std::to_string(maj) + "." + std::to_string(mnr);
+  char hex[32];
+  snprintf(hex, sizeof hex, "%016llx", (unsigned long long)fnv1a(key_src));
+  std::string dir = cache_dir();
+  std::string path = dir + "/" + hex + ".cubin";
+  if (use_cache && read_file(path, cubin)) return true;
+  nvrtcProgram prog;
+  if (nvrtcCreateProgram(&prog, src.c_str(), "rx_program.cu", 0, nullptr, nullptr) != NVRTC_SUCCESS) {
+    log = "nvrtcCreateProgram failed";
+    return false;
+  }
+  std::vector<const char *> ov;
+  for (auto &o : opts) ov.push_back(o.c_str());
+  nvrtcResult r = nvrtcCompileProgram(prog, (int)ov.size(), ov.data());
+  size_t ls = 0;
+  nvrtcGetProgramLogSize(prog, &ls);
+  if (ls > 1) {
+    log.resize(ls);
+    nvrtcGetProgramLog(prog, &log[0]);
+  }
+  if (r != NVRTC_SUCCESS) {
+    nvrtcDestroyProgram(&prog);
+    return false;
+  }
+  size_t cs = 0;
+  nvrtcGetCUBINSize(prog, &cs);
+  cubin.resize(cs);
+  nvrtcGetCUBIN(prog, &cubin[0]);
+  nvrtcDestroyProgram(&prog);
+  if (use_cache) {
+    mkdirs(dir);
+    write_file_atomic(path, cubin);
+  }
+  return true;
+}
+
+}  // namespace
+
+// ---------------------------------------------------------------------------
+// program
+// ---------------------------------------------------------------------------
+struct RxModule {
+  int g_begin = 0, g_end = 0;  // group range
+  int ns_max = 1, nr_max = 1;
+  bool any_state = false;
+  std::string source;
+  std::string cubin;
+  // loaded (device-specific)
+  int device = -1;
+  CUmodule mod = nullptr;
+  CUfunction pass1 = nullptr, fixup = nullptr;
+};
+
+struct rx_program {
+  rx::CompiledSet cs;
+  std::vector<RxModule> mods;
+  uint32_t n_regex = 0;
+  uint32_t state_words = 0;
+  uint32_t lookback = 0, lookahead = 0;
+  std::string all_source;
+  std::string info;
+  std::mutex mu;
+};
+
+extern "C" {
+
+const char *rx_last_error(void) { return g_last_error.c_str(); }
+
+uint32_t rx_num_regex(const rx_program *p) { return p ? p->n_regex : 0; }
+uint32_t rx_num_groups(const rx_program *p) { return p ? (uint32_t)p->cs.groups.size() : 0; }
+uint32_t rx_max_lookback(const rx_program *p) { return p ? p->lookback : 0; }
+uint32_t rx_max_lookahead(const rx_program *p) { return p ? p->lookahead : 0; }
+size_t rx_boundary_bytes(const rx_program *p) { return p ? 4 * (size_t)std::max<uint32_t>(p->state_words, 1) : 0; }
+const char *rx_program_source(const rx_program *p) { return p ? p->all_source.c_str() : ""; }
+const char *rx_program_info(const rx_program *p) { return p ? p->info.c_str() : ""; }
+
+void rx_free(rx_program *p) {
+  if (!p) return;
+  Drv &d = drv();
+  for (auto &m : p->mods)
+    if (m.mod && d.ok) {
+      int cur = -1;
+      cudaGetDevice(&cur);
+      if (cur != m.device) cudaSetDevice(m.device);
+      d.ModuleUnload(m.mod);
+      if (cur != m.device && cur >= 0) cudaSetDevice(cur);
+    }
+  delete p;
+}
+
+rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, uint32_t n_patterns,
+                     const rx_options *opt, rx_program **out, rx_error *err) {
+  if (!out || (n_patterns && (!patterns || !pattern_lens))) return fail(RX_EINVAL, "null argument");
+  *out = nullptr;
+  rx_options o;
+  memset(&o, 0, sizeof o);
+  if (opt) o = *opt;
+  rx::LowerOptions lo;
+  lo.interval = o.interval == 0 ? 8 : (o.interval == UINT32_MAX ? 0 : (int)o.interval);
+  if (o.flags & RX_F_NO_GUARDS) lo.interval = 0;
+  lo.rebalance = !(o.flags & RX_F_NO_REBALANCE);
+  int max_regs = o.max_regs ? (int)o.max_regs : 128;
+
+  auto *p = new rx_program();
+  p->n_regex = n_patterns;
+  p->cs.irs.resize(n_patterns);
+  for (uint32_t i = 0; i < n_patterns; ++i) {
+    std::string pat(patterns[i], pattern_lens[i]);
+    rx::ParseError pe;
+    rx::AstP ast = rx::parse_regex(pat, pe);
+    if (!ast || pe.code) {
+      if (err) {
+        err->pattern_index = i;
+        err->byte_offset = (uint32_t)pe.at;
+        snprintf(err->msg, sizeof err->msg, "%s", pe.msg.c_str());
+      }
+      delete p;
+      return fail((rx_status)pe.code, "pattern " + std::to_string(i) + ": " + pe.msg);
+    }
+    if (rx::ast_expanded_size(*ast) > 20000) {
+      if (err) {
+        err->pattern_index = i;
+        err->byte_offset = 0;
+        snprintf(err->msg, sizeof err->msg, "expansion too large");
+      }
+      delete p;
+      return fail(RX_ETOOBIG, "pattern " + std::to_string(i) + ": expansion too large");
+    }
+    rx::lower_regex(*ast, lo, p->cs.irs[i]);
+    std::string why;
+    if (!rx::analyze_regex(p->cs.irs[i], why)) {
+      delete p;
+      return fail(RX_EUNSUPPORTED, why);
+    }
+  }
+  std::string why;
+  if (!rx::plan_groups(p->cs, (int)o.group_size, (int)o.words_per_lane, why)) {
+    if (err) {
+      err->pattern_index = 0;
+      err->byte_offset = 0;
+      snprintf(err->msg, sizeof err->msg, "%s", why.c_str());
+    }
+    delete p;
+    return fail(RX_ETOOBIG, why);
+  }
+  // modules: split groups for parallel NVRTC compiles
+  int G = (int)p->cs.groups.size();
+  size_t total = 0;
+  for (auto &ir : p->cs.irs) total += ir.n_instr;
+  int nmod = (int)std::min<size_t>((size_t)G, std::max<size_t>(1, (size_t)G / 2));
+  unsigned hw = std::max(1u, std::thread::hardware_concurrency());
+  nmod = std::min<int>(nmod, (int)std::max(1u, hw) * 2);
+  if (nmod < 1) nmod = 1;
+  uint32_t sbase = 0;
+  for (int m = 0; m < nmod; ++m) {
+    RxModule mm;
+    mm.g_begin = (int)((long long)G * m / nmod);
+    mm.g_end = (int)((long long)G * (m + 1) / nmod);
+    p->mods.push_back(mm);
+  }
+  std::ostringstream info;
+  for (int gi = 0; gi < G; ++gi) {
+    auto &g = p->cs.groups[gi];
+    info << "group " << gi << ": regexes=" << g.regexes.size() << " K=" << g.K << " Lw=" << g.Lw << " Rw=" << g.Rw
+         << " Bw=" << g.Bw << " slots=" << g.nslots << "\n";
+    p->lookback = std::max<uint32_t>(p->lookback, 32u * (uint32_t)g.Lw);
+    p->lookahead = std::max<uint32_t>(p->lookahead, 32u * (uint32_t)g.Rw);
+  }
+  for (auto &mm : p->mods) {
+    // this module's groups, with global slot bases / regex ids
+    mm.source = rx::emit_program_source_range(p->cs, mm.g_begin, mm.g_end, sbase);
+    for (int gi = mm.g_begin; gi < mm.g_end; ++gi) {
+      mm.ns_max = std::max(mm.ns_max, p->cs.groups[gi].nslots);
+      mm.nr_max = std::max<int>(mm.nr_max, (int)p->cs.groups[gi].regexes.size());
+      if (p->cs.groups[gi].nslots > 0) mm.any_state = true;
+      sbase += (uint32_t)p->cs.groups[gi].nslots;
+    }
+  }
+  p->state_words = sbase;
+  for (uint32_t i = 0; i < n_patterns; ++i) info << "regex " << i << ":\n" << rx::dump_ir(p->cs.irs[i]);
+  p->info = info.str();
+  // NVRTC (parallel over modules)
+  std::vector<std::string> logs(p->mods.size());
+  std::vector<int> okv(p->mods.size(), 0);
+  bool use_cache = !(o.flags & RX_F_NO_CACHE);
+  {
+    std::vector<std::thread> th;
+    std::atomic<size_t> next{0};
+    size_t nthreads = std::min<size_t>(p->mods.size(), hw);
+    for (size_t t = 0; t < nthreads; ++t)
+      th.emplace_back([&] {
+        for (;;) {
+          size_t m = next++;
+          if (m >= p->mods.size()) break;
+          okv[m] = nvrtc_compile(p->mods[m].source, max_regs, use_cache, p->mods[m].cubin, logs[m]) ? 1 : 0;
+        }
+      });
+    for (auto &t : th) t.join();
+  }
+  for (size_t m = 0; m < p->mods.size(); ++m) {
+    p->all_source += p->mods[m].source;
+    if (!okv[m]) {
+      std::string head = logs[m].substr(0, 240);
+      if (err) {
+        err->pattern_index = 0;
+        err->byte_offset = 0;
+        snprintf(err->msg, sizeof err->msg, "%s", head.c_str());
+      }
+      std::string full = logs[m];
+      delete p;
+      return fail(RX_EJIT, "NVRTC: " + full.substr(0, 4000));
+    }
+  }
+  *out = p;
+  return RX_OK;
+}
+
+}  // extern "C"
+
+// ---------------------------------------------------------------------------
+// launch
+// ---------------------------------------------------------------------------
+namespace {
+
+struct RxParamsHost {  // must mirror RxParams in rx_device.cuh
+  const unsigned char *in;
+  long long avail_lo, avail_hi;
+  long long valid_lo, valid_hi;
+  long long len;
+  long long gofs;
+  unsigned long long *counts;
+  unsigned long long *digests;
+  unsigned int *dense;
+  unsigned long long pitch;
+  unsigned int *status;
+  unsigned int *seg_state;
+  const unsigned int *st_in;
+  unsigned int *st_out;
+  const unsigned int *st_assumed;
+  int sw;
+  int nseg_max;
+  int aligned;
+  int mode;
+  int accumulate;
+};
+
+rx_status ensure_loaded(rx_program *p, int &device) {
+  Drv &d = drv();
+  if (cudaGetDevice(&device) != cudaSuccess) return fail(RX_ECUDA, "no CUDA device");
+  if (!d.ok) return fail(RX_ECUDA, d.why);
+  std::lock_guard<std::mutex> lk(p->mu);
+  for (auto &m : p->mods) {
+    if (m.mod && m.device == device) continue;
+    if (m.mod) return fail(RX_EINVAL, "program was loaded on another device; compile one program per device");
+    cudaFree(nullptr);  // make the primary context current
+    CUresult r = d.ModuleLoadData(&m.mod, m.cubin.data());
+    if (r != CUDA_SUCCESS) return fail(RX_ECUDA, "cuModuleLoadData failed: " + std::to_string((int)r));
+    if (d.ModuleGetFunction(&m.pass1, m.mod, "rx_pass1") != CUDA_SUCCESS ||
+        d.ModuleGetFunction(&m.fixup, m.mod, "rx_fixup") != CUDA_SUCCESS)
+      return fail(RX_ECUDA, "kernel symbols missing");
+    m.device = device;
+  }
+  return RX_OK;
+}
+
+constexpr int kWarpsPerBlock = 4;
+
+rx_status launch(RxModule &m, CUfunction f, long long warps, const RxParamsHost &prm, cudaStream_t s) {
+  Drv &d = drv();
+  if (warps <= 0) return RX_OK;
+  long long blocks = (warps + kWarpsPerBlock - 1) / kWarpsPerBlock;
+  if (blocks > 0x7fffffffLL) return fail(RX_EINVAL, "grid too large");
+  unsigned smem = (unsigned)(kWarpsPerBlock * 3 * m.nr_max * sizeof(unsigned long long));
+  if (smem > 48 * 1024) d.FuncSetAttribute(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)smem);
+  RxParamsHost local = prm;
+  void *args[] = {&local};
+  CUresult r = d.LaunchKernel(f, (unsigned)blocks, 1, 1, 32 * kWarpsPerBlock, 1, 1, smem, (CUstream)s, args, nullptr);
+  if (r != CUDA_SUCCESS) return fail(RX_ECUDA, "cuLaunchKernel failed: " + std::to_string((int)r));
+  return RX_OK;
+}
+
+long long div_up(long long a, long long b) { return (a + b - 1) / b; }
+
+rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo_left, uint64_t halo_right,
+              uint64_t gofs, const void *st_in, void *st_out, const void *st_assumed, int accumulate, int mode,
+              cudaStream_t stream, const rx_output *out) {
+  if (!p || !out || !out->d_counts) return fail(RX_EINVAL, "null argument");
+  if (len && !d_input) return fail(RX_EINVAL, "null input");
+  if (out->d_bitstreams && out->pitch_words < (len + 31) / 32) return fail(RX_EINVAL, "pitch_words too small");
+  if ((halo_left != 0 && halo_left < p->lookback) || (halo_right != 0 && halo_right < p->lookahead))
+    return fail(RX_EINVAL, "halo smaller than rx_max_lookback / rx_max_lookahead");
+  int device = -1;
+  rx_status s = ensure_loaded(p, device);
+  if (s != RX_OK) return s;
+  const uint32_t n = p->n_regex;
+  if (!accumulate && mode != 2) {
+    if (n && cudaMemsetAsync(out->d_counts, 0, 8ull * n, stream) != cudaSuccess) return fail(RX_ECUDA, "memset");
+    if (n && out->d_digests && cudaMemsetAsync(out->d_digests, 0, 16ull * n, stream) != cudaSuccess)
+      return fail(RX_ECUDA, "memset");
+    if (n && out->d_bitstreams &&
+        cudaMemsetAsync(out->d_bitstreams, 0, 4ull * n * out->pitch_words, stream) != cudaSuccess)
+      return fail(RX_ECUDA, "memset");
+    if (out->d_status && cudaMemsetAsync(out->d_status, 0, 4, stream) != cudaSuccess) return fail(RX_ECUDA, "memset");
+  }
+  RxParamsHost prm;
+  memset(&prm, 0, sizeof prm);
+  prm.in = d_input;
+  prm.avail_lo = -(long long)halo_left;
+  prm.avail_hi = (long long)(len + halo_right);
+  // valid stream bytes: a chunk's halo holds real bytes; the stream start
+  // (no halo) has none before position 0
+  prm.valid_lo = -(long long)halo_left;
+  prm.valid_hi = (long long)(len + halo_right);
+  prm.len = (long long)len;
+  prm.gofs = (long long)gofs;
+  prm.counts = (unsigned long long *)out->d_counts;
+  prm.digests = (unsigned long long *)out->d_digests;
+  prm.dense = out->d_bitstreams;
+  prm.pitch = out->pitch_words;
+  prm.status = out->d_status;
+  prm.st_in = (const unsigned int *)st_in;
+  prm.st_out = (unsigned int *)st_out;
+  prm.st_assumed = (const unsigned int *)st_assumed;
+  prm.aligned = (((uintptr_t)d_input) & 15) == 0 ? 1 : 0;
+  prm.accumulate = accumulate;
+  static unsigned int dummy_status_host = 0;
+  (void)dummy_status_host;
+  unsigned int *status_scratch = nullptr;
+  if (!prm.status) {
+    if (cudaMallocAsync((void **)&status_scratch, 4, stream) != cudaSuccess) return fail(RX_ENOMEM, "status");
+    cudaMemsetAsync(status_scratch, 0, 4, stream);
+    prm.status = status_scratch;
+  }
+  const long long len_words = div_up((long long)len, 32);
+  const int G = (int)p->cs.groups.size();
+  if (mode == 2) {
+    prm.mode = 2;
+    prm.sw = 1 << 30;
+    prm.nseg_max = 1;
+    for (auto &m : p->mods) {
+      if (!m.any_state) continue;
+      prm.seg_state = nullptr;
+      s = launch(m, m.fixup, m.g_end - m.g_begin, prm, stream);
+      if (s != RX_OK) return s;
+    }
+    if (status_scratch) cudaFreeAsync(status_scratch, stream);
+    return RX_OK;
+  }
+  // segments: enough warps to fill the GPU several times over
+  long long max_nwin = 0;
+  for (auto &g : p->cs.groups) max_nwin = std::max(max_nwin, div_up(len_words, g.Bw));
+  const long long target_warps = 148LL * 16 * 4;
+  long long sw = std::max<long long>(4, div_up(max_nwin * G, target_warps));
+  long long nseg_max = std::max<long long>(1, div_up(max_nwin, sw));
+  prm.sw = (int)std::min<long long>(sw, 1 << 30);
+  prm.nseg_max = (int)nseg_max;
+  prm.mode = 0;
+  for (auto &m : p->mods) {
+    int mg = m.g_end - m.g_begin;
+    unsigned int *seg_state = nullptr;
+    size_t bytes = 4ull * (size_t)nseg_max * (size_t)mg * (size_t)std::max(1, m.ns_max);
+    if (m.any_state) {
+      if (cudaMallocAsync((void **)&seg_state, bytes, stream) != cudaSuccess) return fail(RX_ENOMEM, "seg_state");
+    }
+    prm.seg_state = seg_state;
+    prm.mode = 0;
+    s = launch(m, m.pass1, nseg_max * mg, prm, stream);
+    if (s != RX_OK) return s;
+    if (m.any_state) {
+      prm.mode = 1;
+      s = launch(m, m.fixup, mg, prm, stream);
+      if (s != RX_OK) return s;
+      cudaFreeAsync(seg_state, stream);
+    }
+  }
+  if (status_scratch) cudaFreeAsync(status_scratch, stream);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(RX_ECUDA, cudaGetErrorString(e));
+  return RX_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+rx_status rx_match(const rx_program *p, const uint8_t *d_input, uint64_t len, void *stream, const rx_output *out) {
+  return run(const_cast<rx_program *>(p), d_input, len, 0, 0, 0, nullptr, nullptr, nullptr, 0, 0,
+             (cudaStream_t)stream, out);
+}
+
+rx_status rx_match_chunk(const rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo_left,
+                         uint64_t halo_right, uint64_t global_offset, const void *d_state_in, void *d_state_out,
+                         int accumulate, void *stream, const rx_output *out) {
+  return run(const_cast<rx_program *>(p), d_input, len, halo_left, halo_right, global_offset, d_state_in,
+             d_state_out, nullptr, accumulate, 0, (cudaStream_t)stream, out);
+}
+
+rx_status rx_rematch_chunk(const rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo_left,
+                           uint64_t halo_right, uint64_t global_offset, const void *d_state_assumed,
+                           const void *d_state_true, void *d_state_out, void *stream, const rx_output *out) {
+  return run(const_cast<rx_program *>(p), d_input, len, halo_left, halo_right, global_offset, d_state_true,
+             d_state_out, d_state_assumed, 1, 2, (cudaStream_t)stream, out);
+}
+
+}  // extern "C"

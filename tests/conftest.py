@@ -6,6 +6,9 @@ import pytest
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 if ROOT not in sys.path:
     sys.path.insert(0, ROOT)
+# JIT cubins are cached in-tree so that programs compiled here are not
+# recompiled on the GPU box (the snapshot carries .rxcache/).
+os.environ.setdefault("RX_CACHE_DIR", os.path.join(ROOT, ".rxcache"))
 
 
 def pytest_configure(config):
