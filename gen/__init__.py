@@ -6,4 +6,5 @@ suites (Table 1; inputs of P:L431), per the recipes in
 DESIGN.md Sec. "Input recipe" / SURVEY.md Sec. 8(d).  Both the oracle side
 (tests, bench cpu_baseline) and the CUDA side (tests, bench) consume it.
 """
-from .workloads import CONFIGS, fuzz_pattern, fuzz_text, make_config, tiny_input, tiny_patterns  # noqa: F401
+from .workloads import (CONFIGS, fuzz_pattern, fuzz_text, make_config, snort_input, snort_patterns,  # noqa: F401
+                        tiny_input, tiny_patterns)

@@ -160,3 +160,239 @@ CONFIGS["tiny"] = {
     "len": 65536,
     "desc": "tiny: 4 regexes over 64 KiB synthetic ASCII (seed 1)",
 }
+
+
+# ---------------------------------------------------------------------------
+# token-based pattern builder: every token renders as regex text and can
+# sample a member string (for planting matches)
+# ---------------------------------------------------------------------------
+_SPECIAL = set(b".^$*+?()[]{}|\\")
+
+
+def _lit_regex(bs: bytes) -> bytes:
+    out = bytearray()
+    for c in bs:
+        if c in _SPECIAL:
+            out += b"\\" + bytes([c])
+        elif 0x20 <= c < 0x7F:
+            out.append(c)
+        else:
+            out += b"\\x%02x" % c
+    return bytes(out)
+
+
+class _Tok:
+    """regex text + a sampler of member strings."""
+
+    def __init__(self, text: bytes, sampler):
+        self.text = text
+        self.sample = sampler
+
+
+def _lit(bs: bytes) -> _Tok:
+    return _Tok(_lit_regex(bs), lambda rng, bs=bs: bs)
+
+
+_CLASSES = {
+    rb"\d": bytes(range(0x30, 0x3A)),
+    rb"\s": b" \t\r\n\f\v",
+    rb"[^\r\n]": bytes(c for c in range(256) if c not in (10, 13)),
+    rb"[A-Za-z0-9]": bytes(range(0x30, 0x3A)) + bytes(range(0x41, 0x5B)) + bytes(range(0x61, 0x7B)),
+    rb"[a-z]": bytes(range(0x61, 0x7B)),
+    rb"[0-9a-f]": bytes(range(0x30, 0x3A)) + bytes(range(0x61, 0x67)),
+    rb".": bytes(c for c in range(256) if c != 10),
+    rb"[^\x00]": bytes(range(1, 256)),
+    rb"\w": bytes(range(0x30, 0x3A)) + bytes(range(0x41, 0x5B)) + bytes(range(0x61, 0x7B)) + b"_",
+}
+
+
+def _quantified(body_text: bytes, body_sample, lo: int, hi: int, qtext: bytes) -> _Tok:
+    def s(rng, lo=lo, hi=hi):
+        n = int(rng.integers(lo, (hi if hi >= 0 else lo + 4) + 1))
+        return b"".join(body_sample(rng) for _ in range(n))
+    return _Tok(body_text + qtext, s)
+
+
+def _class_tok(rng, name=None, quant=True, max_m=64) -> _Tok:
+    names = list(_CLASSES)
+    name = name or names[int(rng.integers(0, len(names)))]
+    members = _CLASSES[name]
+    one = (lambda r, m=members: bytes([m[int(r.integers(0, len(m)))]]))
+    if not quant:
+        return _Tok(name, one)
+    q = rng.random()
+    if q < 0.30:
+        return _quantified(name, one, 1, -1, b"+")
+    if q < 0.55:
+        return _quantified(name, one, 0, -1, b"*")
+    if q < 0.65:
+        return _quantified(name, one, 0, 1, b"?")
+    n = int(rng.integers(0, 9))
+    m = n + int(rng.integers(0, max(1, max_m - n)))
+    m = min(m, max_m)
+    if rng.random() < 0.3:
+        return _quantified(name, one, n, n, b"{%d}" % n)
+    return _quantified(name, one, n, m, b"{%d,%d}" % (n, m))
+
+
+def _alt_tok(words) -> _Tok:
+    text = b"(" + b"|".join(_lit_regex(w) for w in words) + b")"
+    return _Tok(text, lambda rng, w=words: w[int(rng.integers(0, len(w)))])
+
+
+_SNORT_WORDS = [b"GET", b"POST", b"HEAD", b"/cgi-bin/", b"cmd.exe", b"/etc/passwd", b"admin", b"login", b"SELECT",
+                b"union", b"<script>", b".php", b"?id=", b"User-Agent:", b"Content-Length:", b"Host:", b"Cookie:",
+                b"/bin/sh", b"wget ", b"eval(", b"base64_decode", b"%2e%2e%2f", b"../", b"\\x90\\x90", b"HTTP/1.",
+                b"Authorization: Basic ", b"filename=", b"boundary=", b".exe", b"document.cookie", b"onload=",
+                b"javascript:", b"/admin/", b"password=", b"username=", b"action=", b"Referer:", b"PUT", b"DELETE",
+                b"/index.", b"xp_cmdshell", b"exec(", b"system(", b"Accept-Language:", b"Content-Type:"]
+_SNORT_ALTS = [[b"GET", b"POST", b"HEAD"], [b"/", b"\\"], [b"admin", b"root", b"user"],
+               [b"select", b"union", b"insert"], [b"http", b"https", b"ftp"], [b"%20", b"+", b" "]]
+_WORD_ALPHA = b"abcdefghijklmnopqrstuvwxyzABCDEFGHIJKLMNOPQRSTUVWXYZ0123456789_-/.=&%"
+
+
+def _snort_literal(rng) -> bytes:
+    r = rng.random()
+    if r < 0.45:
+        w = _SNORT_WORDS[int(rng.integers(0, len(_SNORT_WORDS)))]
+        return w.replace(b"\\x90", b"\x90")
+    if r < 0.85:
+        n = int(rng.integers(3, 13))
+        return bytes(_WORD_ALPHA[int(i)] for i in rng.integers(0, len(_WORD_ALPHA), size=n))
+    n = int(rng.integers(2, 7))  # binary signature bytes
+    return bytes(rng.integers(0, 256, size=n, dtype=np.uint8))
+
+
+def _group_star(rng) -> _Tok:
+    """A non-CC star (lowered to a while loop, P:L147 / Listing 3)."""
+    r = rng.random()
+    if r < 0.4:
+        sep = bytes([b"/.-_&;"[int(rng.integers(0, 6))]])
+        body = _Tok(_lit_regex(sep) + rb"[a-z0-9]+", lambda g, s=sep: s + bytes(
+            _WORD_ALPHA[:36][int(i)] for i in g.integers(0, 36, size=int(g.integers(1, 5)))))
+    elif r < 0.7:
+        body = _Tok(rb"%[0-9a-f]{2}", lambda g: b"%" + bytes(b"0123456789abcdef"[int(i)] for i in g.integers(0, 16, 2)))
+    else:
+        w = _snort_literal(rng)[:4] or b"ab"
+        body = _Tok(_lit_regex(w), lambda g, w=w: w)
+    q = b"*" if rng.random() < 0.6 else b"+"
+    lo = 0 if q == b"*" else 1
+    return _quantified(b"(?:" + body.text + b")", body.sample, lo, -1, q)
+
+
+def _lognormal_len(rng, mean, sd, lo=4, hi=None):
+    s2 = np.log(1 + (sd / mean) ** 2)
+    mu = np.log(mean) - s2 / 2
+    v = float(rng.lognormal(mu, np.sqrt(s2)))
+    v = max(lo, v)
+    if hi:
+        v = min(v, hi)
+    return int(round(v))
+
+
+def snort_patterns(n: int = 1000, seed: int = 2):
+    """Snort-like set (Table 1 Snort: 1,873 regexes, length mean 50.5, SD 41.5,
+    P:L394; ~2.5 while loops per regex).  Returns (patterns, samplers)."""
+    rng = np.random.default_rng(seed)
+    pats, samplers = [], []
+    for _ in range(n):
+        target = _lognormal_len(rng, 50.5, 41.5, lo=6, hi=400)
+        toks = [_lit(_snort_literal(rng))]
+        size = len(toks[0].text)
+        while size < target:
+            r = rng.random()
+            if r < 0.60:
+                t = _lit(_snort_literal(rng))
+            elif r < 0.80:
+                t = _class_tok(rng)
+            elif r < 0.85:
+                t = _alt_tok(_SNORT_ALTS[int(rng.integers(0, len(_SNORT_ALTS)))])
+            else:
+                t = _group_star(rng)
+            toks.append(t)
+            size += len(t.text)
+        pats.append(b"".join(t.text for t in toks))
+        samplers.append(lambda g, toks=toks: b"".join(t.sample(g) for t in toks))
+    return pats, samplers
+
+
+def _text_pool(rng, n: int, vocab) -> np.ndarray:
+    words = rng.integers(0, len(vocab), size=n // 4)
+    out = b"".join(vocab[int(i)] for i in words)
+    return np.frombuffer(out[:n], dtype=np.uint8)
+
+
+_HTTP_VOCAB = [b"GET ", b"POST ", b"/index.html", b" HTTP/1.1\r\n", b"Host: www.example.com\r\n",
+               b"User-Agent: Mozilla/5.0 (X11; Linux x86_64)\r\n", b"Accept: */*\r\n", b"Connection: keep-alive\r\n",
+               b"Cookie: session=", b"&", b"=", b"id", b"page", b"user", b"the ", b"and ", b"of ", b"to ", b"data",
+               b"/images/", b".png", b".js", b"Content-Type: text/html\r\n", b"\r\n", b"q=search+terms",
+               b"lang=en", b"static", b"api/v1/", b"json", b"200 OK", b"<html>", b"<div class=\"", b"\">",
+               b"</div>", b"var x = ", b"function", b"(", b")", b";", b"0123", b"4567", b"89"]
+
+
+def _fill_records(rng, length, kinds, probs, sources, rec_max=1460):
+    """Stream of records of length U(0, rec_max); each record draws its bytes
+    from sources[kind] at a random offset."""
+    out = np.empty(length, dtype=np.uint8)
+    pos = 0
+    chunk = 1 << 22
+    while pos < length:
+        nrec = chunk // (rec_max // 2) + 2
+        lens = rng.integers(0, rec_max + 1, size=nrec)
+        kind = rng.choice(kinds, size=nrec, p=probs)
+        ends = np.cumsum(lens)
+        take = int(min(length - pos, ends[-1]))
+        nrec_used = int(np.searchsorted(ends, take, side="left")) + 1
+        lens, kind = lens[:nrec_used], kind[:nrec_used]
+        starts = np.concatenate([[0], np.cumsum(lens)[:-1]])
+        rec_id = np.repeat(np.arange(nrec_used), lens)[:take]
+        local = np.arange(take) - starts[rec_id]
+        seg = np.zeros(take, dtype=np.uint8)
+        for k, src in enumerate(sources):
+            m = kind[rec_id] == k
+            if not m.any():
+                continue
+            offs = rng.integers(0, src.size, size=nrec_used)
+            idx = (offs[rec_id[m]] + local[m]) % src.size
+            seg[m] = src[idx]
+        out[pos:pos + take] = seg
+        pos += take
+    return out
+
+
+def _plant(rng, buf: np.ndarray, samplers, every: int):
+    n = buf.size
+    k = max(1, n // every)
+    for _ in range(k):
+        s = samplers[int(rng.integers(0, len(samplers)))](rng)
+        if not s or len(s) >= n:
+            continue
+        at = int(rng.integers(0, n - len(s)))
+        buf[at:at + len(s)] = np.frombuffer(s, dtype=np.uint8)
+
+
+def snort_input(length: int = 256 << 20, seed: int = 2, patterns_seed: int = 2, n_patterns: int = 1000):
+    """Packet payloads: records of 0-1460 B, 50% HTTP-like text, 30% uniform
+    random bytes, 20% base64-ish; members of L(r) of 10% of the regexes
+    planted about once per 64 KiB."""
+    rng = np.random.default_rng(seed * 7919 + 1)
+    pool = min(length, 8 << 20) + 1
+    text = _text_pool(rng, pool, _HTTP_VOCAB)
+    rnd = rng.integers(0, 256, size=pool, dtype=np.uint8)
+    b64a = np.frombuffer(b"ABCDEFGHIJKLMNOPQRSTUVWXYZabcdefghijklmnopqrstuvwxyz0123456789+/", dtype=np.uint8)
+    b64 = b64a[rng.integers(0, 64, size=pool)]
+    buf = _fill_records(rng, length, [0, 1, 2], [0.5, 0.3, 0.2], [text, rnd, b64])
+    _, samplers = snort_patterns(n_patterns, patterns_seed)
+    chosen = [samplers[i] for i in rng.choice(len(samplers), size=max(1, len(samplers) // 10), replace=False)]
+    _plant(rng, buf, chosen, 64 << 10)
+    return buf
+
+
+CONFIGS["snort"] = {
+    "patterns": lambda n=1000, seed=2: snort_patterns(n, seed)[0],
+    "input": lambda length=256 << 20, seed=2: snort_input(length, seed),
+    "pattern_kw": ("n",),
+    "input_kw": ("length",),
+    "len": 256 << 20,
+    "desc": "Snort-like: 1,000 regexes over 256 MiB synthetic packet payloads (seed 2)",
+}

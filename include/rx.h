@@ -87,6 +87,8 @@ uint32_t rx_max_lookback(const rx_program *p);
 uint32_t rx_max_lookahead(const rx_program *p);
 /* Bytes of boundary state (MatchStar carries, forwarded loop tails). */
 size_t rx_boundary_bytes(const rx_program *p);
+/* Number of this library's kernels one rx_match launches (pass 1 + fix-up). */
+uint32_t rx_kernels_per_match(const rx_program *p);
 /* The generated CUDA C source of the program (NUL-terminated, owned by p). */
 const char *rx_program_source(const rx_program *p);
 /* Human-readable IR / per-group geometry dump (owned by p). */

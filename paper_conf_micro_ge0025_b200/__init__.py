@@ -23,7 +23,7 @@ RX_F_NO_REBALANCE, RX_F_NO_GUARDS, RX_F_NO_CACHE = 1, 2, 4
 
 EXPORTED = ["rx_compile", "rx_free", "rx_num_regex", "rx_num_groups", "rx_max_lookback", "rx_max_lookahead",
             "rx_boundary_bytes", "rx_program_source", "rx_program_info", "rx_match", "rx_match_chunk",
-            "rx_rematch_chunk", "rx_last_error"]
+            "rx_rematch_chunk", "rx_last_error", "rx_kernels_per_match"]
 
 
 class RxError(RuntimeError):
@@ -64,7 +64,7 @@ def load_library():
         lib.rx_compile.argtypes = [vp, vp, u32, ctypes.POINTER(_Options), ctypes.POINTER(vp), ctypes.POINTER(_Error)]
         lib.rx_compile.restype = ctypes.c_int
         lib.rx_free.argtypes = [vp]
-        for f in ("rx_num_regex", "rx_num_groups", "rx_max_lookback", "rx_max_lookahead"):
+        for f in ("rx_num_regex", "rx_num_groups", "rx_max_lookback", "rx_max_lookahead", "rx_kernels_per_match"):
             getattr(lib, f).argtypes = [vp]
             getattr(lib, f).restype = u32
         lib.rx_boundary_bytes.argtypes = [vp]
@@ -148,6 +148,10 @@ class Program:
     @property
     def lookahead(self) -> int:
         return int(self._lib.rx_max_lookahead(self._h))
+
+    @property
+    def kernels_per_match(self) -> int:
+        return int(self._lib.rx_kernels_per_match(self._h))
 
     @property
     def boundary_bytes(self) -> int:

@@ -4,6 +4,10 @@
 // straight-line per-group program, the loop/prologue/epilogue template is the
 // hand-written rx_device.cuh).
 //
+// The emitted code is flat per-word scalar C (u32 variables, intrinsics):
+// each IR value of K words per lane becomes K registers; NVVM compiles flat
+// code an order of magnitude faster than template-per-op code.
+//
 // Character classes (Fig. 2a) are emitted as a reduced ordered BDD
 // over the basis streams, MSB (paper b0) first: every node is one mux /
 // and / or / andnot, which ptxas packs into LOP3s.
@@ -26,28 +30,87 @@ struct TabKey {
   }
 };
 
-// truth table helpers: a table at `level` has 2^level meaningful bits
 static bool tab_bit(const uint64_t *w, int i) { return (w[i >> 6] >> (i & 63)) & 1; }
 
 struct RegexEmitter {
   std::ostringstream &os;
   const RegexIR &ir;
   int K;
-  int rloc;        // member index in the group
-  int slot_base;   // first state slot of this regex in the group
+  int rloc;       // member index in the group
+  int slot_base;  // first state slot of this regex in the group
   std::vector<std::map<TabKey, std::string>> cc_scope;
   std::vector<std::map<std::vector<uint64_t>, std::string>> set_scope;
   int tmp = 0;
-  std::string V;
 
   RegexEmitter(std::ostringstream &o, const RegexIR &r, int k, int rl, int sb)
-      : os(o), ir(r), K(k), rloc(rl), slot_base(sb) {
-    V = "V<" + std::to_string(K) + ">";
-  }
+      : os(o), ir(r), K(k), rloc(rl), slot_base(sb) {}
 
   std::string ind(int n) { return std::string(2 * n, ' '); }
   std::string nv(int id) { return "n" + std::to_string(rloc) + "_" + std::to_string(id); }
   std::string fresh() { return "t" + std::to_string(rloc) + "_" + std::to_string(tmp++); }
+  // word i of a vector value; "#0" / "#1" are the constant streams
+  std::string W(const std::string &b, int i) {
+    if (b == "#0") return "0u";
+    if (b == "#1") return "0xffffffffu";
+    return b + "w" + std::to_string(i);
+  }
+  std::string widx(int i) { return "(int)(" + std::to_string(K) + "u * lane + " + std::to_string(i) + "u)"; }
+
+  void decl(int in, const std::string &dst, const std::function<std::string(int)> &e, bool cst = true) {
+    for (int i = 0; i < K; ++i) os << ind(in) << (cst ? "const u32 " : "u32 ") << W(dst, i) << " = " << e(i) << ";\n";
+  }
+  void assign(int in, const std::string &dst, const std::function<std::string(int)> &e) {
+    for (int i = 0; i < K; ++i) os << ind(in) << W(dst, i) << " = " << e(i) << ";\n";
+  }
+  std::string any(const std::string &b) {
+    std::string o;
+    for (int i = 0; i < K; ++i) o += (i ? " | " : "") + W(b, i);
+    return "__any_sync(RX_FULL, (" + o + ") != 0u)";
+  }
+  // word (global index - q) of b, for word i of this lane
+  std::string up(const std::string &b, int q, int i) {
+    int src = i - q;
+    if (src >= 0) return W(b, src);
+    int d = (-src + K - 1) / K;
+    int reg = ((src % K) + K) % K;
+    return "__shfl_up_sync(RX_FULL, " + W(b, reg) + ", " + std::to_string(d) + ")";
+  }
+  std::string down(const std::string &b, int q, int i) {
+    int src = i + q;
+    int d = src / K, reg = src % K;
+    if (d == 0) return W(b, reg);
+    return "__shfl_down_sync(RX_FULL, " + W(b, reg) + ", " + std::to_string(d) + ")";
+  }
+  // Advance (paper "S >> n"): out[p] = in[p - n]
+  void adv(int in, const std::string &dst, const std::string &a, int n) {
+    int Q = n / 32, R = n % 32;
+    if (R == 0) {
+      decl(in, dst, [&](int i) { return up(a, Q, i); });
+      return;
+    }
+    decl(in, dst, [&](int i) {
+      return "__funnelshift_l(" + up(a, Q + 1, i) + ", " + up(a, Q, i) + ", " + std::to_string(R) + ")";
+    });
+  }
+  // Lookahead (paper "S << n"): out[p] = in[p + n]
+  void look(int in, const std::string &dst, const std::string &a, int n) {
+    int Q = n / 32, R = n % 32;
+    if (R == 0) {
+      decl(in, dst, [&](int i) { return down(a, Q, i); });
+      return;
+    }
+    decl(in, dst, [&](int i) {
+      return "__funnelshift_r(" + down(a, Q, i) + ", " + down(a, Q + 1, i) + ", " + std::to_string(R) + ")";
+    });
+  }
+  // broadcast of word `wexpr` (runtime) of b
+  std::string extract(const std::string &b, const std::string &wexpr) {
+    if (K == 1) return "__shfl_sync(RX_FULL, " + W(b, 0) + ", " + wexpr + ")";
+    std::string sel = W(b, K - 1);
+    for (int i = K - 2; i >= 0; --i)
+      sel = "((" + wexpr + ") % " + std::to_string(K) + " == " + std::to_string(i) + " ? " + W(b, i) + " : " + sel + ")";
+    return "__shfl_sync(RX_FULL, " + sel + ", (" + wexpr + ") / " + std::to_string(K) + ")";
+  }
 
   // --- character classes -------------------------------------------------
   std::string bdd(int level, const uint64_t *tab, int in) {
@@ -72,18 +135,19 @@ struct RegexEmitter {
       if (tab_bit(tab, i + h)) t1[i >> 6] |= 1ull << (i & 63);
     }
     std::string f0 = bdd(level - 1, t0, in), f1 = bdd(level - 1, t1, in);
-    std::string b = "c.bit[" + std::to_string(level - 1) + "]";
-    std::string e;
     if (f0 == f1) return f0;
-    if (f0 == "#0" && f1 == "#1") e = b;
-    else if (f0 == "#1" && f1 == "#0") e = "vnot(" + b + ")";
-    else if (f0 == "#0") e = "vand(" + b + ", " + f1 + ")";
-    else if (f1 == "#0") e = "vandn(" + f0 + ", " + b + ")";
-    else if (f1 == "#1") e = "vor(" + b + ", " + f0 + ")";
-    else if (f0 == "#1") e = "vornot(" + f1 + ", " + b + ")";
-    else e = "vsel(" + b + ", " + f1 + ", " + f0 + ")";
+    std::string b = "b" + std::to_string(level - 1);
     std::string t = fresh();
-    os << ind(in) << "const " << V << " " << t << " = " << e << ";\n";
+    decl(in, t, [&](int i) {
+      std::string B = W(b, i), F0 = W(f0, i), F1 = W(f1, i);
+      if (f0 == "#0" && f1 == "#1") return B;
+      if (f0 == "#1" && f1 == "#0") return "~" + B;
+      if (f0 == "#0") return "(" + B + " & " + F1 + ")";
+      if (f1 == "#0") return "(" + F0 + " & ~" + B + ")";
+      if (f1 == "#1") return "(" + B + " | " + F0 + ")";
+      if (f0 == "#1") return "(" + F1 + " | ~" + B + ")";
+      return "((" + B + " & " + F1 + ") | (~" + B + " & " + F0 + "))";
+    });
     cc_scope.back()[key] = t;
     return t;
   }
@@ -96,13 +160,13 @@ struct RegexEmitter {
     }
     std::string e = bdd(8, s.w, in);
     std::string out;
-    if (e == "#0") out = "vzero<" + std::to_string(K) + ">()";
-    else if (e == "#1") out = "c.vm";
+    if (e == "#0") out = "#0";
+    else if (e == "#1") out = "vm";
     else if (s.has(0)) {
       // a class containing 0x00 would match the zero padding: mask with the
       // valid-data stream (reading c9)
       out = fresh();
-      os << ind(in) << "const " << V << " " << out << " = vand(" << e << ", c.vm);\n";
+      decl(in, out, [&](int i) { return W(e, i) + " & " + W("vm", i); });
     } else {
       out = e;
     }
@@ -113,7 +177,6 @@ struct RegexEmitter {
   void push() { cc_scope.emplace_back(); set_scope.emplace_back(); }
   void pop() { cc_scope.pop_back(); set_scope.pop_back(); }
 
-  // state slots read by stateful sites inside a block (for guard pending tests)
   void collect_slots(int block, std::vector<int> &out) {
     for (int id : ir.blocks[block].nodes) {
       const Node &n = ir.nodes[id];
@@ -129,75 +192,125 @@ struct RegexEmitter {
     for (int id : ir.blocks[b].nodes) node(id, in, first);
   }
 
+  // MatchStar in match-end form: ((((X + C) ^ C) | X) & C), X masked to
+  // words >= aw; long add = per-lane K-word add + generate/propagate ballots
+  // + carry-lookahead on lane masks; carry in at word aw, carry into word
+  // aw+cw out.
+  void mstar(int in, const std::string &dst, const std::string &X, const std::string &C, int aw,
+             const std::string &cin, const std::string &cout_lhs, bool accumulate) {
+    std::string p = fresh();
+    std::string I = ind(in);
+    decl(in, dst, [&](int) { return std::string("0u"); }, false);
+    os << I << "{\n";
+    std::string J = ind(in + 1);
+    for (int i = 0; i < K; ++i)
+      os << J << "const u32 " << p << "x" << i << " = " << widx(i) << " >= " << aw << " ? " << W(X, i) << " : 0u;\n";
+    os << J << "u32 " << p << "c = 0u; bool " << p << "p = true;\n";
+    for (int i = 0; i < K; ++i) {
+      os << J << "u32 " << p << "s" << i << ";\n";
+      os << J << "{ const unsigned long long t = (unsigned long long)" << p << "x" << i << " + " << W(C, i) << " + ("
+         << widx(i) << " == " << aw << " ? (" << cin << ") : 0u) + " << p << "c; " << p << "s" << i
+         << " = (u32)t; " << p << "c = (u32)(t >> 32); " << p << "p = " << p << "p && (" << p << "s" << i
+         << " == 0xffffffffu); }\n";
+    }
+    os << J << "const u32 " << p << "G = __ballot_sync(RX_FULL, " << p << "c != 0u);\n";
+    os << J << "const u32 " << p << "P = __ballot_sync(RX_FULL, " << p << "p);\n";
+    os << J << "const u32 " << p << "A = " << p << "G | " << p << "P;\n";
+    os << J << "const u32 " << p << "v = (" << p << "A + " << p << "G) ^ " << p << "A ^ " << p << "G;\n";
+    os << J << "u32 " << p << "l = (" << p << "v >> lane) & 1u;\n";
+    for (int i = 0; i < K; ++i) {
+      os << J << "{ const unsigned long long t = (unsigned long long)" << p << "s" << i << " + " << p << "l; " << p
+         << "s" << i << " = (u32)t; " << p << "l = (u32)(t >> 32); }\n";
+      os << J << W(dst, i) << " = ((" << p << "s" << i << " ^ " << W(C, i) << ") | " << p << "x" << i << ") & "
+         << W(C, i) << ";\n";
+      os << J << "const u32 " << p << "qw" << i << " = " << p << "s" << i << " ^ " << p << "x" << i << " ^ "
+         << W(C, i) << ";\n";
+    }
+    os << J << "const int " << p << "e = " << aw << " + cw;\n";
+    os << J << "const u32 " << p << "top = (" << p << "G >> 31) | ((" << p << "P >> 31) & (" << p << "v >> 31) & 1u);\n";
+    os << J << "const u32 " << p << "in = "
+       << extract(p + "q", "(" + p + "e < " + std::to_string(32 * K) + " ? " + p + "e : 0)") << " & 1u;\n";
+    os << J << cout_lhs << (accumulate ? " |= " : " = ") << "(" << p << "e >= " << 32 * K << " ? " << p << "top : " << p
+       << "in);\n";
+    os << I << "}\n";
+  }
+
   void node(int id, int in, const std::string &first) {
     const Node &n = ir.nodes[id];
     std::string I = ind(in);
-    auto A = [&] { return nv(n.a); };
-    auto B = [&] { return nv(n.b); };
+    auto val = [&](int x) -> std::string {  // Zero / Ones operands fold to constants
+      if (x < 0) return "";
+      if (ir.nodes[x].op == Op::Zero) return "#0";
+      if (ir.nodes[x].op == Op::Ones) return "#1";
+      return nv(x);
+    };
+    std::string A = val(n.a), B = val(n.b);
     switch (n.op) {
-      case Op::Zero: os << I << "const " << V << " " << nv(id) << " = vzero<" << K << ">();\n"; break;
-      case Op::Ones: os << I << "const " << V << " " << nv(id) << " = vones<" << K << ">();\n"; break;
-      case Op::Fr: break;  // declared by the loop
+      case Op::Zero: case Op::Ones: case Op::Fr: break;
       case Op::CC: {
         std::string e = cc(ir.sets[n.cc], in);
-        os << I << "const " << V << " " << nv(id) << " = " << e << ";\n";
+        decl(in, nv(id), [&](int i) { return W(e, i); });
         break;
       }
-      case Op::And: os << I << "const " << V << " " << nv(id) << " = vand(" << A() << ", " << B() << ");\n"; break;
-      case Op::Or: os << I << "const " << V << " " << nv(id) << " = vor(" << A() << ", " << B() << ");\n"; break;
-      case Op::Xor: os << I << "const " << V << " " << nv(id) << " = vxor(" << A() << ", " << B() << ");\n"; break;
-      case Op::AndNot: os << I << "const " << V << " " << nv(id) << " = vandn(" << A() << ", " << B() << ");\n"; break;
+      case Op::And: decl(in, nv(id), [&](int i) { return W(A, i) + " & " + W(B, i); }); break;
+      case Op::Or: decl(in, nv(id), [&](int i) { return W(A, i) + " | " + W(B, i); }); break;
+      case Op::Xor: decl(in, nv(id), [&](int i) { return W(A, i) + " ^ " + W(B, i); }); break;
+      case Op::AndNot: decl(in, nv(id), [&](int i) { return W(A, i) + " & ~" + W(B, i); }); break;
       case Op::Adv:
         if (n.loop >= 0) {
-          os << I << "const " << V << " " << nv(id) << " = advf(c, " << A() << ", " << n.aw << ", " << first
-             << " ? " << st(n.slot) << " : 0u, " << nst(n.slot) << ");\n";
+          // forwarded advance inside a loop body: inject the previous
+          // window's operand word at aw-1 (first iteration only), collect
+          // the word at aw-1+cw for the next window
+          std::string t = fresh();
+          decl(in, t, [&](int i) {
+            return W(A, i) + " | (" + widx(i) + " == " + std::to_string(n.aw - 1) + " && " + first + " ? " + st(n.slot) +
+                   " : 0u)";
+          });
+          os << I << nst(n.slot) << " |= " << extract(t, std::to_string(n.aw - 1) + " + cw") << ";\n";
+          adv(in, nv(id), t, n.k);
         } else {
-          os << I << "const " << V << " " << nv(id) << " = vadv<" << n.k << ">(" << A() << ");\n";
+          adv(in, nv(id), A, n.k);
         }
         break;
-      case Op::Look: os << I << "const " << V << " " << nv(id) << " = vlook<" << n.k << ">(" << A() << ");\n"; break;
+      case Op::Look: look(in, nv(id), A, n.k); break;
       case Op::MStar:
-        if (n.loop >= 0) {
-          std::string co = fresh();
-          os << I << "u32 " << co << ";\n";
-          os << I << "const " << V << " " << nv(id) << " = mstar(c, " << A() << ", " << B() << ", " << n.aw << ", "
-             << first << " ? " << st(n.slot) << " : 0u, " << co << ");\n";
-          os << I << nst(n.slot) << " |= " << co << ";\n";
-        } else {
-          os << I << "const " << V << " " << nv(id) << " = mstar(c, " << A() << ", " << B() << ", " << n.aw << ", "
-             << st(n.slot) << ", " << nst(n.slot) << ");\n";
-        }
+        if (n.loop >= 0)
+          mstar(in, nv(id), A, B, n.aw, "(" + first + " ? " + st(n.slot) + " : 0u)", nst(n.slot), true);
+        else
+          mstar(in, nv(id), A, B, n.aw, st(n.slot), nst(n.slot), false);
         break;
       case Op::Loop: {
         // while-fixpoint of Fig. 2e / Listing 3
         std::string L = std::to_string(rloc) + "_" + std::to_string(id);
         std::string acc = "acc" + L, fr = "fr" + L, fst = "first" + L, it = "it" + L, nw = "nw" + L;
-        os << I << V << " " << nv(id) << ";\n" << I << "{\n";
+        std::string aw = std::to_string(n.aw);
+        decl(in, nv(id), [&](int) { return std::string("0u"); }, false);
+        os << I << "{\n";
         // k=1: the operand holds ends of r (acc starts with them);
         // k=0: the operand holds prefix ends (the first frontier only)
         if (n.k == 1) {
-          os << I << "  " << V << " " << acc << " = vmask_ge(c, " << A() << ", " << n.aw << ");\n";
-          os << I << "  " << V << " " << fr << " = " << acc << ";\n";
+          decl(in + 1, acc, [&](int i) { return widx(i) + " >= " + aw + " ? " + W(A, i) + " : 0u"; }, false);
+          decl(in + 1, fr, [&](int i) { return W(acc, i); }, false);
         } else {
-          os << I << "  " << V << " " << acc << " = vzero<" << K << ">();\n";
-          os << I << "  " << V << " " << fr << " = vmask_ge(c, " << A() << ", " << n.aw << ");\n";
+          decl(in + 1, acc, [&](int) { return std::string("0u"); }, false);
+          decl(in + 1, fr, [&](int i) { return widx(i) + " >= " + aw + " ? " + W(A, i) + " : 0u"; }, false);
         }
         os << I << "  bool " << fst << " = " << (first.empty() ? "true" : first) << ";\n";
         os << I << "  u32 " << it << " = 0u;\n";
         os << I << "  while (true) {\n";
-        os << I << "    const " << V << " " << nv(n.fr) << " = " << fr << ";\n";
+        decl(in + 2, nv(n.fr), [&](int i) { return W(fr, i); });
         push();
         block(n.sub, in + 2, fst);
         pop();
-        os << I << "    const " << V << " " << nw << " = vmask_ge(c, vandn(" << nv(n.res) << ", " << acc << "), "
-           << n.aw << ");\n";
-        os << I << "    if (!vany(" << nw << ")) break;\n";
-        os << I << "    " << acc << " = vor(" << acc << ", " << nw << ");\n";
-        os << I << "    " << fr << " = " << nw << ";\n";
+        std::string R = val(n.res);
+        decl(in + 2, nw, [&](int i) { return widx(i) + " >= " + aw + " ? (" + W(R, i) + " & ~" + W(acc, i) + ") : 0u"; });
+        os << I << "    if (!" << any(nw) << ") break;\n";
+        assign(in + 2, acc, [&](int i) { return W(acc, i) + " | " + W(nw, i); });
+        assign(in + 2, fr, [&](int i) { return W(nw, i); });
         os << I << "    " << fst << " = false;\n";
-        os << I << "    if (++" << it << " > RX_LOOP_CAP) { if (c.lane == 0) atomicOr(c.status, 1u); break; }\n";
+        os << I << "    if (++" << it << " > RX_LOOP_CAP) { if (lane == 0) atomicOr(c.status, 1u); break; }\n";
         os << I << "  }\n";
-        os << I << "  " << nv(id) << " = " << acc << ";\n";
+        assign(in + 1, nv(id), [&](int i) { return W(acc, i); });
         os << I << "}\n";
         break;
       }
@@ -208,12 +321,13 @@ struct RegexEmitter {
         collect_slots(n.sub, slots);
         std::string pend;
         for (size_t i = 0; i < slots.size(); ++i) pend += (i ? " | " : "") + st(slots[i]);
-        os << I << V << " " << nv(id) << " = vzero<" << K << ">();\n";
-        os << I << "if (vany(" << A() << ")" << (pend.empty() ? "" : " || ((" + pend + ") != 0u)") << ") {\n";
+        decl(in, nv(id), [&](int) { return std::string("0u"); }, false);
+        os << I << "if (" << any(A) << (pend.empty() ? "" : " || ((" + pend + ") != 0u)") << ") {\n";
         push();
         block(n.sub, in + 1, first);
         pop();
-        os << I << "  " << nv(id) << " = " << nv(n.res) << ";\n";
+        std::string R = val(n.res);
+        assign(in + 1, nv(id), [&](int i) { return W(R, i); });
         os << I << "}\n";
         break;
       }
@@ -226,7 +340,16 @@ struct RegexEmitter {
     block(0, 3, "");
     pop();
     const Node &o = ir.nodes[ir.out];
-    if (o.op != Op::Zero) os << "      emit(c, " << rloc << ", " << nv(ir.out) << ");\n";
+    if (o.op != Op::Zero) {
+      std::string R = nv(ir.out);
+      std::string m;
+      for (int i = 0; i < K; ++i) m += (i ? " | " : "") + ("(" + W(R, i) + " & c.cm[" + std::to_string(i) + "])");
+      os << "      if (c.want_dense || __any_sync(RX_FULL, (" << m << ") != 0u)) {\n";
+      os << "        V<" << K << "> ov;\n";
+      for (int i = 0; i < K; ++i) os << "        ov.w[" << i << "] = " << W(R, i) << ";\n";
+      os << "        rx_emit<" << K << ">(c, " << rloc << ", ov);\n";
+      os << "      }\n";
+    }
     os << "    }\n";
   }
 };
@@ -235,19 +358,30 @@ struct RegexEmitter {
 
 extern const char *kDevicePrelude;
 
-std::string emit_program_source_range(CompiledSet &cs, int g_begin, int g_end, uint32_t sbase0) {
-  std::ostringstream os;
-  os << kDevicePrelude << "\n// ===================== generated program =====================\n";
-  int G = g_end - g_begin;
-  int nsmax = 0, nrmax = 1, sbase = (int)sbase0;
-  for (int gi = g_begin; gi < g_end; ++gi) {
-    nsmax = std::max(nsmax, cs.groups[gi].nslots);
-    nrmax = std::max(nrmax, (int)cs.groups[gi].regexes.size());
+static void layout(const CompiledSet &cs, int &nsmax, int &nrmax) {
+  nsmax = 1;
+  nrmax = 1;
+  for (auto &g : cs.groups) {
+    nsmax = std::max(nsmax, g.nslots);
+    nrmax = std::max(nrmax, (int)g.regexes.size());
   }
-  if (nsmax < 1) nsmax = 1;
-  os << "#define RX_NG " << G << "\n#define RX_NSMAX " << nsmax << "\n#define RX_NRMAX " << nrmax << "\n";
-  for (int gi = 0; gi < G; ++gi) {
-    Group &g = cs.groups[g_begin + gi];
+}
+
+// One relocatable compilation unit per group (NVRTC -rdc): the group's
+// traits, its program body, and the two non-inlined entry functions
+// rx_seg_<g> (pass 1 over one segment) and rx_fix_<g> (carry fix-up).
+// Compile time stays linear in the number of groups; nvJitLink links the
+// units with the kernel unit into one module.
+std::string emit_group_unit(CompiledSet &cs, int gi) {
+  std::ostringstream os;
+  os << kDevicePrelude << "\n// ===================== generated group " << gi << " =====================\n";
+  int nsmax, nrmax;
+  layout(cs, nsmax, nrmax);
+  int G = (int)cs.groups.size();
+  int sbase = 0;
+  for (int h = 0; h < gi; ++h) sbase += cs.groups[h].nslots;
+  {
+    Group &g = cs.groups[gi];
     os << "__device__ const int rx_rid_" << gi << "[" << g.regexes.size() << "] = {";
     for (size_t i = 0; i < g.regexes.size(); ++i) os << (i ? "," : "") << g.regexes[i];
     os << "};\n";
@@ -256,30 +390,53 @@ std::string emit_program_source_range(CompiledSet &cs, int g_begin, int g_end, u
        << ", NR = " << g.regexes.size() << ", SBASE = " << sbase << ", NG = " << G << ", GID = " << gi
        << ", NSMAX = " << nsmax << ";\n";
     os << "  static DEV const int *rid() { return rx_rid_" << gi << "; }\n";
-    os << "  static DEV void body(Ctx<" << g.K << "> &c, const u32 *st, u32 *nst) {\n";
+    os << "  static DEV void body(Ctx<" << g.K << "> &c, const u32 (&pl)[8][" << g.K
+       << "], const u32 *st, u32 *nst) {\n";
     os << "    (void)st; (void)nst;\n";
+    os << "    const u32 lane = c.lane; const int cw = (int)c.cw; (void)cw;\n";
+    for (int k = 0; k < 8; ++k)
+      for (int i = 0; i < g.K; ++i) os << "    const u32 b" << k << "w" << i << " = pl[" << k << "][" << i << "];\n";
+    for (int i = 0; i < g.K; ++i) os << "    const u32 vmw" << i << " = c.vm[" << i << "];\n";
     for (size_t m = 0; m < g.regexes.size(); ++m) {
       RegexEmitter em(os, cs.irs[g.regexes[m]], g.K, (int)m, g.slot_base[m]);
       em.emit_regex();
     }
     os << "  }\n};\n";
-    // one non-inlined function per group and pass: ptxas compiles each
-    // separately (compile time stays linear in the number of groups)
-    os << "__device__ __noinline__ void rx_seg_" << gi << "(const RxParams &p, int seg, u64 *acc) { rx_run_segment<RxG"
-       << gi << ">(p, seg, acc); }\n";
+    os << "extern \"C\" __device__ __noinline__ void rx_seg_" << gi
+       << "(const RxParams &p, int seg, u64 *acc) { rx_run_segment<RxG" << gi << ">(p, seg, acc); }\n";
     if (g.nslots > 0)
-      os << "__device__ __noinline__ void rx_fix_" << gi << "(const RxParams &p, u64 *acc) { rx_fixup_group<RxG" << gi
-         << ">(p, acc); }\n";
-    sbase += g.nslots;
+      os << "extern \"C\" __device__ __noinline__ void rx_fix_" << gi
+         << "(const RxParams &p, u64 *acc) { rx_fixup_group<RxG" << gi << ">(p, acc); }\n";
   }
+  return os.str();
+}
+
+// The kernel unit: rx_pass1 (warp -> (segment, group), groups of one
+// segment interleaved so that they read the same input region together)
+// and rx_fixup (one warp per stateful group).
+std::string emit_kernel_unit(CompiledSet &cs) {
+  std::ostringstream os;
+  os << kDevicePrelude << "\n// ===================== kernels =====================\n";
+  int nsmax, nrmax;
+  layout(cs, nsmax, nrmax);
+  int G = (int)cs.groups.size();
+  os << "#define RX_NG " << G << "\n#define RX_NSMAX " << nsmax << "\n#define RX_NRMAX " << nrmax << "\n";
+  for (int gi = 0; gi < G; ++gi) {
+    os << "extern \"C\" __device__ void rx_seg_" << gi << "(const RxParams &p, int seg, u64 *acc);\n";
+    if (cs.groups[gi].nslots > 0) os << "extern \"C\" __device__ void rx_fix_" << gi << "(const RxParams &p, u64 *acc);\n";
+  }
+  int g_begin = 0;
   os << "\nextern \"C\" __global__ void __launch_bounds__(128) rx_pass1(const RxParams p) {\n"
         "  extern __shared__ u64 rx_smem[];\n"
         "  const int warp = threadIdx.x >> 5;\n"
         "  u64 *acc = rx_smem + warp * (3 * RX_NRMAX);\n"
         "  const long long wid = (long long)blockIdx.x * (blockDim.x >> 5) + warp;\n"
-        "  const int g = (int)(wid % RX_NG);\n"
-        "  const long long seg = wid / RX_NG;\n"
-        "  if (seg >= p.nseg_max) return;\n"
+        // group-major: the warps of a CTA (and of consecutive CTAs on an SM)
+        // run the same group's code over consecutive segments, so the SM's
+        // instruction caches hold one program at a time
+        "  const int g = (int)(wid / p.nseg_max);\n"
+        "  const long long seg = wid % p.nseg_max;\n"
+        "  if (g >= RX_NG) return;\n"
         "  switch (g) {\n";
   for (int gi = 0; gi < G; ++gi) os << "    case " << gi << ": rx_seg_" << gi << "(p, (int)seg, acc); break;\n";
   os << "    default: break;\n  }\n}\n";

@@ -41,120 +41,14 @@ DEV u32 rx_lane() {
   return l;
 }
 
-template <int K> DEV V<K> vzero() { V<K> r;
-#pragma unroll
-  for (int i = 0; i < K; ++i) r.w[i] = 0u;
-  return r; }
-template <int K> DEV V<K> vones() { V<K> r;
-#pragma unroll
-  for (int i = 0; i < K; ++i) r.w[i] = RX_FULL;
-  return r; }
-template <int K> DEV V<K> vand(const V<K> &a, const V<K> &b) { V<K> r;
-#pragma unroll
-  for (int i = 0; i < K; ++i) r.w[i] = a.w[i] & b.w[i];
-  return r; }
-template <int K> DEV V<K> vor(const V<K> &a, const V<K> &b) { V<K> r;
-#pragma unroll
-  for (int i = 0; i < K; ++i) r.w[i] = a.w[i] | b.w[i];
-  return r; }
-template <int K> DEV V<K> vxor(const V<K> &a, const V<K> &b) { V<K> r;
-#pragma unroll
-  for (int i = 0; i < K; ++i) r.w[i] = a.w[i] ^ b.w[i];
-  return r; }
-template <int K> DEV V<K> vandn(const V<K> &a, const V<K> &b) { V<K> r;  // a & ~b
-#pragma unroll
-  for (int i = 0; i < K; ++i) r.w[i] = a.w[i] & ~b.w[i];
-  return r; }
-template <int K> DEV V<K> vornot(const V<K> &a, const V<K> &b) { V<K> r;  // a | ~b
-#pragma unroll
-  for (int i = 0; i < K; ++i) r.w[i] = a.w[i] | ~b.w[i];
-  return r; }
-template <int K> DEV V<K> vnot(const V<K> &a) { V<K> r;
-#pragma unroll
-  for (int i = 0; i < K; ++i) r.w[i] = ~a.w[i];
-  return r; }
-// s ? t : f, bitwise (one LOP3)
-template <int K> DEV V<K> vsel(const V<K> &s, const V<K> &t, const V<K> &f) { V<K> r;
-#pragma unroll
-  for (int i = 0; i < K; ++i) r.w[i] = (s.w[i] & t.w[i]) | (~s.w[i] & f.w[i]);
-  return r; }
-
-template <int K> DEV bool vany(const V<K> &a) {
-  u32 o = 0;
-#pragma unroll
-  for (int i = 0; i < K; ++i) o |= a.w[i];
-  return __any_sync(RX_FULL, o != 0u);
-}
-
-// word shift toward higher positions by Q words (word j <- word j-Q); the
-// words shifted in at the window's left edge are garbage (inside lb).
-template <int Q, int K> DEV V<K> wshl(const V<K> &x) {
-  V<K> r;
-#pragma unroll
-  for (int i = 0; i < K; ++i) {
-    const int src = i - Q;
-    const int d = src >= 0 ? 0 : (-src + K - 1) / K;
-    const int reg = ((src % K) + K) % K;
-    r.w[i] = d == 0 ? x.w[reg] : __shfl_up_sync(RX_FULL, x.w[reg], d);
-  }
-  return r;
-}
-// word shift toward lower positions by Q words (word j <- word j+Q)
-template <int Q, int K> DEV V<K> wshr(const V<K> &x) {
-  V<K> r;
-#pragma unroll
-  for (int i = 0; i < K; ++i) {
-    const int src = i + Q;
-    const int d = src / K;
-    const int reg = src % K;
-    r.w[i] = d == 0 ? x.w[reg] : __shfl_down_sync(RX_FULL, x.w[reg], d);
-  }
-  return r;
-}
-
-// Advance (paper "S >> N", Fig. 2b): out[p] = x[p - N]
-template <int N, int K> DEV V<K> vadv(const V<K> &x) {
-  if constexpr (N == 0) {
-    return x;
-  } else if constexpr (N % 32 == 0) {
-    return wshl<N / 32>(x);
-  } else {
-    constexpr int Q = N / 32, R = N % 32;
-    V<K> y;
-    if constexpr (Q == 0) y = x; else y = wshl<Q>(x);
-    V<K> z = wshl<Q + 1>(x);
-    V<K> r;
-#pragma unroll
-    for (int i = 0; i < K; ++i) r.w[i] = __funnelshift_l(z.w[i], y.w[i], R);
-    return r;
-  }
-}
-// Lookahead (paper "S << N", from Shift Rebalancing): out[p] = x[p + N]
-template <int N, int K> DEV V<K> vlook(const V<K> &x) {
-  if constexpr (N == 0) {
-    return x;
-  } else if constexpr (N % 32 == 0) {
-    return wshr<N / 32>(x);
-  } else {
-    constexpr int Q = N / 32, R = N % 32;
-    V<K> y;
-    if constexpr (Q == 0) y = x; else y = wshr<Q>(x);
-    V<K> z = wshr<Q + 1>(x);
-    V<K> r;
-#pragma unroll
-    for (int i = 0; i < K; ++i) r.w[i] = __funnelshift_r(y.w[i], z.w[i], R);
-    return r;
-  }
-}
-
 // ---------------------------------------------------------------------------
-// window context
+// window context (scalars only: the 8 basis streams live in a register array
+// of the segment loop and are passed to the body separately)
 // ---------------------------------------------------------------------------
 template <int K>
 struct Ctx {
-  V<K> bit[8];  // basis streams: bit[k] = bit k of each byte (paper b_{7-k}; b0 = MSB)
-  V<K> vm;      // positions holding real stream bytes
-  V<K> cm;      // committed positions of this window inside [0, len)
+  u32 vm[K];    // positions holding real stream bytes
+  u32 cm[K];    // committed positions of this window inside [0, len)
   u32 lane;
   u32 cw;       // committed words of this window
   u64 *acc;     // per-warp shared accumulators [NR][3] (count, d1, d2)
@@ -168,78 +62,10 @@ struct Ctx {
   u32 *status;
 };
 
-template <int K> DEV V<K> vmask_ge(const Ctx<K> &c, const V<K> &x, int aw) {
-  V<K> r;
-#pragma unroll
-  for (int i = 0; i < K; ++i) r.w[i] = ((int)(c.lane * K + i) >= aw) ? x.w[i] : 0u;
-  return r;
-}
-template <int K> DEV void vinject(const Ctx<K> &c, V<K> &x, int w, u32 t) {
-#pragma unroll
-  for (int i = 0; i < K; ++i)
-    if ((int)(c.lane * K + i) == w) x.w[i] |= t;
-}
-// value of word w (runtime) broadcast to the warp
-template <int K> DEV u32 vextract(const Ctx<K> &c, const V<K> &x, int w) {
-  u32 v = x.w[0];
-#pragma unroll
-  for (int i = 1; i < K; ++i)
-    if ((w % K) == i) v = x.w[i];
-  return __shfl_sync(RX_FULL, v, w / K);
-}
-
-// Forwarded Advance by 1 inside a while-loop body: the operand's word aw-1
-// receives the previous window's value (tin; only in the first iteration),
-// and the value at word aw-1+cw is OR-accumulated for the next window.
-template <int K> DEV V<K> advf(const Ctx<K> &c, V<K> x, int aw, u32 tin, u32 &tout) {
-  vinject(c, x, aw - 1, tin);
-  tout |= vextract(c, x, aw - 1 + (int)c.cw);
-  return vadv<1>(x);
-}
-
-// MatchStar in match-end form: ends of X C* = ((((X + C) ^ C) | X) & C),
-// X subset of C (Parabix MatchStar [24], SURVEY App.A-6).  Long-stream add:
-// per-lane K-word add, generate/propagate ballots, carry-lookahead as a
-// 32-bit add on lane masks, carry-in injected at word aw, carry into word
-// aw+cw returned for the next window.
-template <int K> DEV V<K> mstar(const Ctx<K> &c, V<K> X, const V<K> &C, int aw, u32 cin, u32 &cout) {
-  X = vmask_ge(c, X, aw);
-  u32 s[K];
-  u32 carry = 0u;
-  bool allones = true;
-#pragma unroll
-  for (int i = 0; i < K; ++i) {
-    u32 ci = ((int)(c.lane * K + i) == aw) ? cin : 0u;
-    u64 t = (u64)X.w[i] + (u64)C.w[i] + (u64)ci + (u64)carry;
-    s[i] = (u32)t;
-    carry = (u32)(t >> 32);
-    allones = allones && (s[i] == RX_FULL);
-  }
-  u32 G = __ballot_sync(RX_FULL, carry != 0u);
-  u32 P = __ballot_sync(RX_FULL, allones);
-  u32 A = G | P;
-  u32 cvec = (A + G) ^ A ^ G;  // bit l = carry into lane l
-  u32 cl = (cvec >> c.lane) & 1u;
-  V<K> r, q;
-#pragma unroll
-  for (int i = 0; i < K; ++i) {
-    u64 t = (u64)s[i] + (u64)cl;
-    s[i] = (u32)t;
-    cl = (u32)(t >> 32);
-    r.w[i] = ((s[i] ^ C.w[i]) | X.w[i]) & C.w[i];
-    q.w[i] = s[i] ^ X.w[i] ^ C.w[i];  // bit b = carry into that bit
-  }
-  // carry into word aw+cw; aw+cw == 32K (a window with no right halo) is
-  // the carry out of the last lane
-  const int ew = aw + (int)c.cw;
-  const u32 top = (G >> 31) | (((P >> 31) & (cvec >> 31)) & 1u);  // g | (p & c_in) of lane 31
-  const u32 inner = vextract(c, q, ew < 32 * K ? ew : 0) & 1u;
-  cout = ew >= 32 * K ? top : inner;
-  return r;
-}
-
 // ---------------------------------------------------------------------------
-// epilogue
+// epilogue (called only when the output has a set bit in the committed
+// range, or when dense output is requested): popcount -> REDUX, digests,
+// dense store
 // ---------------------------------------------------------------------------
 DEV u64 rx_splitmix64(u64 x) {
   u64 z = x + 0x9E3779B97F4A7C15ull;
@@ -254,38 +80,36 @@ DEV u64 rx_warp_sum64(u64 v) {
   return v;
 }
 
-template <int K> DEV void emit(Ctx<K> &c, int r, const V<K> &v) {
+template <int K>
+__device__ __noinline__ void rx_emit(const Ctx<K> c, int r, const V<K> v) {
   u32 m[K];
   u32 any = 0u;
 #pragma unroll
   for (int i = 0; i < K; ++i) {
-    m[i] = v.w[i] & c.cm.w[i];
+    m[i] = v.w[i] & c.cm[i];
     any |= m[i];
   }
   if (c.want_dense) {
     u32 *row = c.dense + (u64)c.rid[r] * c.pitch;
 #pragma unroll
-    for (int i = 0; i < K; ++i) {
-      int j = (int)(c.lane * K + i);
-      i64 aw = c.word0 + j;
-      if (c.cm.w[i] != 0u || (aw >= 0 && j >= 0 && false)) row[aw] = m[i];
-    }
+    for (int i = 0; i < K; ++i)
+      if (c.cm[i] != 0u) row[c.word0 + (i64)(c.lane * K + i)] = m[i];
   }
   if (!__any_sync(RX_FULL, any != 0u)) return;
   u32 cnt = 0;
 #pragma unroll
   for (int i = 0; i < K; ++i) cnt += __popc(m[i]);
-  u32 tot = __reduce_add_sync(RX_FULL, cnt);
+  const u32 tot = __reduce_add_sync(RX_FULL, cnt);
   u64 d1 = 0, d2 = 0;
   if (c.want_digest) {
 #pragma unroll
     for (int i = 0; i < K; ++i) {
       u32 b = m[i];
-      i64 base = c.gofs + (c.word0 + (i64)(c.lane * K + i)) * 32;
+      const i64 base = c.gofs + (c.word0 + (i64)(c.lane * K + i)) * 32;
       while (b) {
-        int t = __ffs(b) - 1;
+        const int t = __ffs(b) - 1;
         b &= b - 1u;
-        u64 p = (u64)(base + t);
+        const u64 p = (u64)(base + t);
         d1 += rx_splitmix64(p);
         d2 += rx_splitmix64(p ^ 0x9E3779B97F4A7C15ull);
       }
@@ -304,15 +128,15 @@ template <int K> DEV void emit(Ctx<K> &c, int r, const V<K> &v) {
 // prologue: load + fused transposition
 // ---------------------------------------------------------------------------
 // 32 bytes x[0..7] (little-endian words) -> 8 basis words: plane[k] bit j =
-// bit k of byte j.
+// bit k of byte j (paper b_{7-k}, b0 = MSB).
 DEV void rx_transpose32(const u32 x[8], u32 plane[8]) {
   // byte transpose: y[r] byte q = byte (8q + r)
   u32 y[8];
 #pragma unroll
   for (int h = 0; h < 2; ++h) {
-    u32 a = x[0 + h], b = x[2 + h], cc = x[4 + h], d = x[6 + h];
-    u32 t0 = __byte_perm(a, b, 0x5140), t1 = __byte_perm(a, b, 0x7362);
-    u32 t2 = __byte_perm(cc, d, 0x5140), t3 = __byte_perm(cc, d, 0x7362);
+    const u32 a = x[0 + h], b = x[2 + h], cc = x[4 + h], d = x[6 + h];
+    const u32 t0 = __byte_perm(a, b, 0x5140), t1 = __byte_perm(a, b, 0x7362);
+    const u32 t2 = __byte_perm(cc, d, 0x5140), t3 = __byte_perm(cc, d, 0x7362);
     y[4 * h + 0] = __byte_perm(t0, t2, 0x5410);
     y[4 * h + 1] = __byte_perm(t0, t2, 0x7632);
     y[4 * h + 2] = __byte_perm(t1, t3, 0x5410);
@@ -321,7 +145,7 @@ DEV void rx_transpose32(const u32 x[8], u32 plane[8]) {
   // 8x8 bit transpose inside each byte lane, across the 8 registers
 #define RX_SWAP(r0, r1, s, m)                   \
   {                                             \
-    u32 t = ((y[r0] >> (s)) ^ y[r1]) & (m);     \
+    const u32 t = ((y[r0] >> (s)) ^ y[r1]) & (m); \
     y[r1] ^= t;                                 \
     y[r0] ^= t << (s);                          \
   }
@@ -355,40 +179,40 @@ struct RxParams {
   int accumulate;           // counts/digests are added to (else the host zeroed them)
 };
 
-template <int K> DEV void rx_load_window(const RxParams &p, Ctx<K> &c, i64 fword) {
+template <int K> DEV void rx_load_window(const RxParams &p, Ctx<K> &c, u32 (&pl)[8][K], i64 fword) {
 #pragma unroll
   for (int i = 0; i < K; ++i) {
-    i64 wi = fword + (i64)(c.lane * K + i);
-    i64 pos = wi * 32;
+    const i64 wi = fword + (i64)(c.lane * K + i);
+    const i64 pos = wi * 32;
     u32 x[8];
     if (p.aligned && pos >= p.avail_lo && pos + 32 <= p.avail_hi) {
       const uint4 *q = reinterpret_cast<const uint4 *>(p.in + pos);
-      uint4 a = __ldg(q), b = __ldg(q + 1);
+      const uint4 a = __ldg(q), b = __ldg(q + 1);
       x[0] = a.x; x[1] = a.y; x[2] = a.z; x[3] = a.w;
       x[4] = b.x; x[5] = b.y; x[6] = b.z; x[7] = b.w;
     } else {
 #pragma unroll
       for (int j = 0; j < 8; ++j) x[j] = 0u;
       for (int j = 0; j < 32; ++j) {
-        i64 ps = pos + j;
+        const i64 ps = pos + j;
         if (ps >= p.avail_lo && ps < p.avail_hi) x[j >> 2] |= (u32)p.in[ps] << (8 * (j & 3));
       }
     }
-    u32 pl[8];
-    rx_transpose32(x, pl);
+    u32 t[8];
+    rx_transpose32(x, t);
 #pragma unroll
-    for (int k = 0; k < 8; ++k) c.bit[k].w[i] = pl[k];
+    for (int k = 0; k < 8; ++k) pl[k][i] = t[k];
     // valid-data mask
-    i64 lo = p.valid_lo - pos, hi = p.valid_hi - pos;  // valid bits [lo, hi) of this word
+    const i64 lo = p.valid_lo - pos, hi = p.valid_hi - pos;  // valid bits [lo, hi) of this word
     u32 m;
     if (lo <= 0 && hi >= 32) m = RX_FULL;
     else if (hi <= 0 || lo >= 32) m = 0u;
     else {
-      u32 a = lo <= 0 ? RX_FULL : (RX_FULL << (u32)lo);
-      u32 b = hi >= 32 ? RX_FULL : (RX_FULL >> (u32)(32 - hi));
+      const u32 a = lo <= 0 ? RX_FULL : (RX_FULL << (u32)lo);
+      const u32 b = hi >= 32 ? RX_FULL : (RX_FULL >> (u32)(32 - hi));
       m = a & b;
     }
-    c.vm.w[i] = m;
+    c.vm[i] = m;
   }
 }
 
@@ -396,29 +220,32 @@ template <int K> DEV void rx_load_window(const RxParams &p, Ctx<K> &c, i64 fword
 template <int K> DEV void rx_commit_mask(const RxParams &p, Ctx<K> &c, int Lw, i64 fword) {
 #pragma unroll
   for (int i = 0; i < K; ++i) {
-    int j = (int)(c.lane * K + i);
+    const int j = (int)(c.lane * K + i);
     u32 m = 0u;
     if (j >= Lw && j < Lw + (int)c.cw) {
-      i64 pos = (fword + j) * 32;
-      i64 hi = p.len - pos;
+      const i64 pos = (fword + j) * 32;
+      const i64 hi = p.len - pos;
       m = hi >= 32 ? RX_FULL : (hi <= 0 ? 0u : (RX_FULL >> (u32)(32 - hi)));
     }
-    c.cm.w[i] = m;
+    c.cm[i] = m;
   }
 }
 
 DEV i64 rx_div_up(i64 a, i64 b) { return (a + b - 1) / b; }
 
-// Runs one group (traits G) over one segment (pass 1).
-template <class G>
-DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc) {
-  constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS > 0 ? G::NS : 1;
-  const i64 len_words = rx_div_up(p.len, 32);
-  const i64 nwin = rx_div_up(len_words, Bw);
-  const i64 w_begin = (i64)seg * p.sw;
-  if (w_begin >= nwin && !(seg == 0)) return;
-  const i64 w_end = w_begin + p.sw < nwin ? w_begin + p.sw : nwin;
-  Ctx<K> c;
+template <class G> DEV void rx_flush(const RxParams &p, const Ctx<G::K> &c) {
+  __syncwarp();
+  for (int r = (int)c.lane; r < G::NR; r += 32) {
+    const int gr = G::rid()[r];
+    if (c.acc[3 * r]) atomicAdd(&p.counts[gr], c.acc[3 * r]);
+    if (p.digests) {
+      if (c.acc[3 * r + 1]) atomicAdd(&p.digests[2 * gr], c.acc[3 * r + 1]);
+      if (c.acc[3 * r + 2]) atomicAdd(&p.digests[2 * gr + 1], c.acc[3 * r + 2]);
+    }
+  }
+}
+
+template <class G> DEV void rx_ctx_init(const RxParams &p, Ctx<G::K> &c, u64 *acc) {
   c.lane = rx_lane();
   c.acc = acc;
   c.dense = p.dense;
@@ -431,6 +258,20 @@ DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc) {
   c.status = p.status;
   for (int r = (int)c.lane; r < 3 * G::NR; r += 32) acc[r] = 0ull;
   __syncwarp();
+}
+
+// Runs one group (traits G) over one segment (pass 1).
+template <class G>
+DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc) {
+  constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS > 0 ? G::NS : 1;
+  const i64 len_words = rx_div_up(p.len, 32);
+  const i64 nwin = rx_div_up(len_words, Bw);
+  const i64 w_begin = (i64)seg * p.sw;
+  if (w_begin >= nwin && seg != 0) return;
+  const i64 w_end = w_begin + p.sw < nwin ? w_begin + p.sw : nwin;
+  Ctx<K> c;
+  rx_ctx_init<G>(p, c, acc);
+  u32 pl[8][K];
   u32 st[NS], nst[NS];
 #pragma unroll
   for (int s = 0; s < NS; ++s) st[s] = (seg == 0 && p.st_in) ? p.st_in[G::SBASE + s] : 0u;
@@ -439,11 +280,11 @@ DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc) {
     const i64 fword = cstart - Lw;
     c.cw = (u32)((len_words - cstart) < Bw ? (len_words - cstart) : Bw);
     c.word0 = fword;
-    rx_load_window(p, c, fword);
+    rx_load_window(p, c, pl, fword);
     rx_commit_mask(p, c, Lw, fword);
 #pragma unroll
     for (int s = 0; s < NS; ++s) nst[s] = 0u;
-    G::body(c, st, nst);
+    G::body(c, pl, st, nst);
 #pragma unroll
     for (int s = 0; s < NS; ++s) st[s] = nst[s];
   }
@@ -458,15 +299,7 @@ DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc) {
       for (int s = 0; s < NS; ++s) p.st_out[G::SBASE + s] = st[s];
     }
   }
-  __syncwarp();
-  for (int r = (int)c.lane; r < G::NR; r += 32) {
-    int gr = G::rid()[r];
-    if (acc[3 * r]) atomicAdd(&p.counts[gr], acc[3 * r]);
-    if (p.digests) {
-      if (acc[3 * r + 1]) atomicAdd(&p.digests[2 * gr], acc[3 * r + 1]);
-      if (acc[3 * r + 2]) atomicAdd(&p.digests[2 * gr + 1], acc[3 * r + 2]);
-    }
-  }
+  rx_flush<G>(p, c);
 }
 
 template <int NS> DEV bool rx_state_eq(const u32 *a, const u32 *b) {
@@ -487,28 +320,14 @@ DEV void rx_fixup_group(const RxParams &p, u64 *acc) {
   const i64 nwin = rx_div_up(len_words, Bw);
   const i64 nseg = rx_div_up(nwin, p.sw);
   Ctx<K> c;
-  c.lane = rx_lane();
-  c.acc = acc;
-  c.dense = p.dense;
-  c.pitch = p.pitch;
-  c.gofs = p.gofs;
-  c.want_digest = p.digests != nullptr;
-  c.rid = G::rid();
-  c.status = p.status;
-  for (int r = (int)c.lane; r < 3 * G::NR; r += 32) acc[r] = 0ull;
-  __syncwarp();
+  rx_ctx_init<G>(p, c, acc);
+  u32 pl[8][K];
   u32 tru[NS], old[NS], t1[NS], t2[NS];
-  if (p.mode == 2) {
 #pragma unroll
-    for (int s = 0; s < NS; ++s) {
-      tru[s] = p.st_in ? p.st_in[G::SBASE + s] : 0u;
-      old[s] = p.st_assumed ? p.st_assumed[G::SBASE + s] : 0u;
-    }
-  } else {
-#pragma unroll
-    for (int s = 0; s < NS; ++s) tru[s] = p.st_in ? p.st_in[G::SBASE + s] : 0u;
+  for (int s = 0; s < NS; ++s) {
+    tru[s] = p.st_in ? p.st_in[G::SBASE + s] : 0u;
+    old[s] = (p.mode == 2 && p.st_assumed) ? p.st_assumed[G::SBASE + s] : 0u;
   }
-  bool changed = false;
   for (i64 seg = 0; seg < nseg; ++seg) {
     const i64 w_begin = seg * p.sw;
     const i64 w_end = w_begin + p.sw < nwin ? w_begin + p.sw : nwin;
@@ -523,24 +342,26 @@ DEV void rx_fixup_group(const RxParams &p, u64 *acc) {
       const i64 fword = cstart - Lw;
       c.cw = (u32)((len_words - cstart) < Bw ? (len_words - cstart) : Bw);
       c.word0 = fword;
-      rx_load_window(p, c, fword);
+      rx_load_window(p, c, pl, fword);
       rx_commit_mask(p, c, Lw, fword);
       // old run: subtract
       c.sign = ~0ull;
       c.want_dense = false;
 #pragma unroll
       for (int s = 0; s < NS; ++s) t1[s] = 0u;
-      G::body(c, old, t1);
+      G::body(c, pl, old, t1);
       // new run: add, rewrite dense words
       c.sign = 1ull;
       c.want_dense = p.dense != nullptr;
 #pragma unroll
       for (int s = 0; s < NS; ++s) t2[s] = 0u;
-      G::body(c, tru, t2);
+      G::body(c, pl, tru, t2);
 #pragma unroll
-      for (int s = 0; s < NS; ++s) { old[s] = t1[s]; tru[s] = t2[s]; }
+      for (int s = 0; s < NS; ++s) {
+        old[s] = t1[s];
+        tru[s] = t2[s];
+      }
       conv = rx_state_eq<NS>(tru, old);
-      changed = true;
     }
     if (conv) {
       if (p.mode == 2) break;  // identical to the caller's run from here on
@@ -554,14 +375,5 @@ DEV void rx_fixup_group(const RxParams &p, u64 *acc) {
       for (int s = 0; s < NS; ++s) p.st_out[G::SBASE + s] = tru[s];
     }
   }
-  (void)changed;
-  __syncwarp();
-  for (int r = (int)c.lane; r < G::NR; r += 32) {
-    int gr = G::rid()[r];
-    if (acc[3 * r]) atomicAdd(&p.counts[gr], acc[3 * r]);
-    if (p.digests) {
-      if (acc[3 * r + 1]) atomicAdd(&p.digests[2 * gr], acc[3 * r + 1]);
-      if (acc[3 * r + 2]) atomicAdd(&p.digests[2 * gr + 1], acc[3 * r + 2]);
-    }
-  }
+  rx_flush<G>(p, c);
 }

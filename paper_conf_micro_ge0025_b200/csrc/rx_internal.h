@@ -128,8 +128,10 @@ struct CompiledSet {
   std::string info;
 };
 
-// CUDA C source of groups [g_begin, g_end) as one module (slot base sbase0).
-std::string emit_program_source_range(CompiledSet &cs, int g_begin, int g_end, uint32_t sbase0);
+// CUDA C sources: one relocatable unit per group + the kernel unit; linked
+// into one module with nvJitLink.
+std::string emit_group_unit(CompiledSet &cs, int gi);
+std::string emit_kernel_unit(CompiledSet &cs);
 bool plan_groups(CompiledSet &cs, int group_size, int force_K, std::string &why);
 
 }  // namespace rx

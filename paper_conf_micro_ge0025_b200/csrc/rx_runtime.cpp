@@ -45,6 +45,11 @@ struct Drv {
                            CUstream, void **, void **) = nullptr;
   CUresult (*FuncSetAttribute)(CUfunction, CUfunction_attribute, int) = nullptr;
   CUresult (*ModuleUnload)(CUmodule) = nullptr;
+  CUresult (*LinkCreate)(unsigned, CUjit_option *, void **, CUlinkState *) = nullptr;
+  CUresult (*LinkAddData)(CUlinkState, CUjitInputType, void *, size_t, const char *, unsigned, CUjit_option *,
+                          void **) = nullptr;
+  CUresult (*LinkComplete)(CUlinkState, void **, size_t *) = nullptr;
+  CUresult (*LinkDestroy)(CUlinkState) = nullptr;
   bool ok = false;
   std::string why;
 };
@@ -62,7 +67,9 @@ Drv &drv() {
               get("cuModuleGetFunction", (void **)&d.ModuleGetFunction) &&
               get("cuLaunchKernel", (void **)&d.LaunchKernel) &&
               get("cuFuncSetAttribute", (void **)&d.FuncSetAttribute) &&
-              get("cuModuleUnload", (void **)&d.ModuleUnload);
+              get("cuModuleUnload", (void **)&d.ModuleUnload) && get("cuLinkCreate", (void **)&d.LinkCreate) &&
+              get("cuLinkAddData", (void **)&d.LinkAddData) && get("cuLinkComplete", (void **)&d.LinkComplete) &&
+              get("cuLinkDestroy", (void **)&d.LinkDestroy);
     d.ok = ok;
     if (!ok) d.why = "CUDA driver entry points unavailable (no GPU / driver?)";
   });
@@ -124,7 +131,7 @@ bool nvrtc_compile(const std::string &src, int max_regs, bool use_cache, std::st
   int maj = 0, mnr = 0;
   nvrtcVersion(&maj, &mnr);
   std::vector<std::string> opts = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo", "-default-device",
-                                   "--maxrregcount=" + std::to_string(max_regs), "-DNDEBUG"};
+                                   "-rdc=true", "--maxrregcount=" + std::to_string(max_regs), "-DNDEBUG"};
   std::string key_src = src;
   for (auto &o : opts) key_src += "\n//" + o;
   key_src += "\n//nvrtc " + std::to_string(maj) + "." + std::to_string(mnr);
@@ -173,7 +180,7 @@ struct RxModule {
   int ns_max = 1, nr_max = 1;
   bool any_state = false;
   std::string source;
-  std::string cubin;
+  std::vector<std::string> units;  // relocatable sm_100a cubins (groups + kernels)
   // loaded (device-specific)
   int device = -1;
   CUmodule mod = nullptr;
@@ -201,6 +208,12 @@ uint32_t rx_max_lookback(const rx_program *p) { return p ? p->lookback : 0; }
 uint32_t rx_max_lookahead(const rx_program *p) { return p ? p->lookahead : 0; }
 size_t rx_boundary_bytes(const rx_program *p) { return p ? 4 * (size_t)std::max<uint32_t>(p->state_words, 1) : 0; }
 const char *rx_program_source(const rx_program *p) { return p ? p->all_source.c_str() : ""; }
+uint32_t rx_kernels_per_match(const rx_program *p) {
+  uint32_t n = 0;
+  if (p)
+    for (auto &m : p->mods) n += 1 + (m.any_state ? 1 : 0);
+  return n;
+}
 const char *rx_program_info(const rx_program *p) { return p ? p->info.c_str() : ""; }
 
 void rx_free(rx_program *p) {
@@ -272,62 +285,49 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
     delete p;
     return fail(RX_ETOOBIG, why);
   }
-  // modules: split groups for parallel NVRTC compiles
+  // one relocatable NVRTC unit per group + the kernel unit, compiled in
+  // parallel and linked into one module by nvJitLink
   int G = (int)p->cs.groups.size();
-  size_t total = 0;
-  for (auto &ir : p->cs.irs) total += ir.n_instr;
-  int nmod = (int)std::min<size_t>((size_t)G, std::max<size_t>(1, (size_t)G / 2));
   unsigned hw = std::max(1u, std::thread::hardware_concurrency());
-  nmod = std::min<int>(nmod, (int)std::max(1u, hw) * 2);
-  if (nmod < 1) nmod = 1;
-  uint32_t sbase = 0;
-  for (int m = 0; m < nmod; ++m) {
-    RxModule mm;
-    mm.g_begin = (int)((long long)G * m / nmod);
-    mm.g_end = (int)((long long)G * (m + 1) / nmod);
-    p->mods.push_back(mm);
-  }
   std::ostringstream info;
+  uint32_t sbase = 0;
+  RxModule mm;
+  mm.g_begin = 0;
+  mm.g_end = G;
   for (int gi = 0; gi < G; ++gi) {
     auto &g = p->cs.groups[gi];
     info << "group " << gi << ": regexes=" << g.regexes.size() << " K=" << g.K << " Lw=" << g.Lw << " Rw=" << g.Rw
          << " Bw=" << g.Bw << " slots=" << g.nslots << "\n";
     p->lookback = std::max<uint32_t>(p->lookback, 32u * (uint32_t)g.Lw);
     p->lookahead = std::max<uint32_t>(p->lookahead, 32u * (uint32_t)g.Rw);
-  }
-  for (auto &mm : p->mods) {
-    // this module's groups, with global slot bases / regex ids
-    mm.source = rx::emit_program_source_range(p->cs, mm.g_begin, mm.g_end, sbase);
-    for (int gi = mm.g_begin; gi < mm.g_end; ++gi) {
-      mm.ns_max = std::max(mm.ns_max, p->cs.groups[gi].nslots);
-      mm.nr_max = std::max<int>(mm.nr_max, (int)p->cs.groups[gi].regexes.size());
-      if (p->cs.groups[gi].nslots > 0) mm.any_state = true;
-      sbase += (uint32_t)p->cs.groups[gi].nslots;
-    }
+    mm.ns_max = std::max(mm.ns_max, g.nslots);
+    mm.nr_max = std::max<int>(mm.nr_max, (int)g.regexes.size());
+    if (g.nslots > 0) mm.any_state = true;
+    sbase += (uint32_t)g.nslots;
   }
   p->state_words = sbase;
   for (uint32_t i = 0; i < n_patterns; ++i) info << "regex " << i << ":\n" << rx::dump_ir(p->cs.irs[i]);
   p->info = info.str();
-  // NVRTC (parallel over modules)
-  std::vector<std::string> logs(p->mods.size());
-  std::vector<int> okv(p->mods.size(), 0);
+  std::vector<std::string> srcs(G + 1), cubins(G + 1), logs(G + 1);
+  for (int gi = 0; gi < G; ++gi) srcs[gi] = rx::emit_group_unit(p->cs, gi);
+  srcs[G] = rx::emit_kernel_unit(p->cs);
+  std::vector<int> okv(G + 1, 0);
   bool use_cache = !(o.flags & RX_F_NO_CACHE);
   {
     std::vector<std::thread> th;
     std::atomic<size_t> next{0};
-    size_t nthreads = std::min<size_t>(p->mods.size(), hw);
+    size_t nthreads = std::min<size_t>(srcs.size(), hw);
     for (size_t t = 0; t < nthreads; ++t)
       th.emplace_back([&] {
         for (;;) {
           size_t m = next++;
-          if (m >= p->mods.size()) break;
-          okv[m] = nvrtc_compile(p->mods[m].source, max_regs, use_cache, p->mods[m].cubin, logs[m]) ? 1 : 0;
+          if (m >= srcs.size()) break;
+          okv[m] = nvrtc_compile(srcs[m], max_regs, use_cache, cubins[m], logs[m]) ? 1 : 0;
         }
       });
     for (auto &t : th) t.join();
   }
-  for (size_t m = 0; m < p->mods.size(); ++m) {
-    p->all_source += p->mods[m].source;
+  for (size_t m = 0; m < srcs.size(); ++m) {
     if (!okv[m]) {
       std::string head = logs[m].substr(0, 240);
       if (err) {
@@ -340,6 +340,9 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
       return fail(RX_EJIT, "NVRTC: " + full.substr(0, 4000));
     }
   }
+  mm.units = std::move(cubins);  // relocatable; linked by the driver at module load
+  for (auto &s : srcs) p->all_source += s;
+  p->mods.push_back(mm);
   *out = p;
   return RX_OK;
 }
@@ -382,8 +385,26 @@ rx_status ensure_loaded(rx_program *p, int &device) {
     if (m.mod && m.device == device) continue;
     if (m.mod) return fail(RX_EINVAL, "program was loaded on another device; compile one program per device");
     cudaFree(nullptr);  // make the primary context current
-    CUresult r = d.ModuleLoadData(&m.mod, m.cubin.data());
-    if (r != CUDA_SUCCESS) return fail(RX_ECUDA, "cuModuleLoadData failed: " + std::to_string((int)r));
+    // link the relocatable units (SASS already: no JIT) into one image
+    char lerr[4096];
+    lerr[0] = 0;
+    CUjit_option lo[] = {CU_JIT_ERROR_LOG_BUFFER, CU_JIT_ERROR_LOG_BUFFER_SIZE_BYTES};
+    void *lv[] = {(void *)lerr, (void *)(uintptr_t)sizeof lerr};
+    CUlinkState ls;
+    CUresult r = d.LinkCreate(2, lo, lv, &ls);
+    if (r != CUDA_SUCCESS) return fail(RX_ECUDA, "cuLinkCreate failed: " + std::to_string((int)r));
+    for (size_t u = 0; u < m.units.size() && r == CUDA_SUCCESS; ++u) {
+      std::string nm = "unit" + std::to_string(u) + ".cubin";
+      r = d.LinkAddData(ls, CU_JIT_INPUT_CUBIN, (void *)m.units[u].data(), m.units[u].size(), nm.c_str(), 0, nullptr,
+                        nullptr);
+    }
+    void *img = nullptr;
+    size_t img_size = 0;
+    if (r == CUDA_SUCCESS) r = d.LinkComplete(ls, &img, &img_size);
+    if (r == CUDA_SUCCESS) r = d.ModuleLoadData(&m.mod, img);
+    d.LinkDestroy(ls);
+    if (r != CUDA_SUCCESS)
+      return fail(RX_ECUDA, "link/load of the program failed: " + std::to_string((int)r) + " " + lerr);
     if (d.ModuleGetFunction(&m.pass1, m.mod, "rx_pass1") != CUDA_SUCCESS ||
         d.ModuleGetFunction(&m.fixup, m.mod, "rx_fixup") != CUDA_SUCCESS)
       return fail(RX_ECUDA, "kernel symbols missing");
