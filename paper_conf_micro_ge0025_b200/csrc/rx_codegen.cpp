@@ -403,10 +403,10 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
     }
     os << "  }\n};\n";
     os << "extern \"C\" __device__ __noinline__ void rx_seg_" << gi
-       << "(const RxParams &p, int seg, u64 *acc) { rx_run_segment<RxG" << gi << ">(p, seg, acc); }\n";
+       << "(const RxParams &p, int seg, u64 *acc, u32 *sst) { rx_run_segment<RxG" << gi << ">(p, seg, acc, sst); }\n";
     if (g.nslots > 0)
       os << "extern \"C\" __device__ __noinline__ void rx_fix_" << gi
-         << "(const RxParams &p, u64 *acc) { rx_fixup_group<RxG" << gi << ">(p, acc); }\n";
+         << "(const RxParams &p, u64 *acc, u32 *sst) { rx_fixup_group<RxG" << gi << ">(p, acc, sst); }\n";
   }
   return os.str();
 }
@@ -422,33 +422,39 @@ std::string emit_kernel_unit(CompiledSet &cs) {
   int G = (int)cs.groups.size();
   os << "#define RX_NG " << G << "\n#define RX_NSMAX " << nsmax << "\n#define RX_NRMAX " << nrmax << "\n";
   for (int gi = 0; gi < G; ++gi) {
-    os << "extern \"C\" __device__ void rx_seg_" << gi << "(const RxParams &p, int seg, u64 *acc);\n";
-    if (cs.groups[gi].nslots > 0) os << "extern \"C\" __device__ void rx_fix_" << gi << "(const RxParams &p, u64 *acc);\n";
+    os << "extern \"C\" __device__ void rx_seg_" << gi << "(const RxParams &p, int seg, u64 *acc, u32 *sst);\n";
+    if (cs.groups[gi].nslots > 0)
+      os << "extern \"C\" __device__ void rx_fix_" << gi << "(const RxParams &p, u64 *acc, u32 *sst);\n";
   }
   int g_begin = 0;
-  os << "\nextern \"C\" __global__ void __launch_bounds__(128) rx_pass1(const RxParams p) {\n"
+  // pass 1: one CTA of 16 warps (the whole SM's register file) runs one
+  // group over 16 consecutive segments in lockstep, so the SM's instruction
+  // caches hold one program at a time
+  os << "\nextern \"C\" __global__ void __launch_bounds__(512, 1) rx_pass1(const RxParams p) {\n"
         "  extern __shared__ u64 rx_smem[];\n"
         "  const int warp = threadIdx.x >> 5;\n"
+        "  const int wpb = blockDim.x >> 5;\n"
+        // shared memory per warp: [3*NRMAX] u64 accumulators, then [4*NSMAX] u32 state
         "  u64 *acc = rx_smem + warp * (3 * RX_NRMAX);\n"
-        "  const long long wid = (long long)blockIdx.x * (blockDim.x >> 5) + warp;\n"
-        // group-major: the warps of a CTA (and of consecutive CTAs on an SM)
-        // run the same group's code over consecutive segments, so the SM's
-        // instruction caches hold one program at a time
-        "  const int g = (int)(wid / p.nseg_max);\n"
-        "  const long long seg = wid % p.nseg_max;\n"
+        "  u32 *sst = reinterpret_cast<u32 *>(rx_smem + wpb * (3 * RX_NRMAX)) + warp * (4 * RX_NSMAX);\n"
+        "  const int cpg = (p.nseg_max + wpb - 1) / wpb;  // CTAs per group\n"
+        "  const int g = (int)(blockIdx.x / cpg);\n"
+        "  const long long seg = (long long)(blockIdx.x % cpg) * wpb + warp;\n"
         "  if (g >= RX_NG) return;\n"
         "  switch (g) {\n";
-  for (int gi = 0; gi < G; ++gi) os << "    case " << gi << ": rx_seg_" << gi << "(p, (int)seg, acc); break;\n";
+  for (int gi = 0; gi < G; ++gi) os << "    case " << gi << ": rx_seg_" << gi << "(p, (int)seg, acc, sst); break;\n";
   os << "    default: break;\n  }\n}\n";
   os << "\nextern \"C\" __global__ void __launch_bounds__(128) rx_fixup(const RxParams p) {\n"
         "  extern __shared__ u64 rx_smem[];\n"
         "  const int warp = threadIdx.x >> 5;\n"
+        "  const int wpb = blockDim.x >> 5;\n"
         "  u64 *acc = rx_smem + warp * (3 * RX_NRMAX);\n"
-        "  const long long g = (long long)blockIdx.x * (blockDim.x >> 5) + warp;\n"
+        "  u32 *sst = reinterpret_cast<u32 *>(rx_smem + wpb * (3 * RX_NRMAX)) + warp * (4 * RX_NSMAX);\n"
+        "  const long long g = (long long)blockIdx.x * wpb + warp;\n"
         "  if (g >= RX_NG) return;\n"
         "  switch ((int)g) {\n";
   for (int gi = 0; gi < G; ++gi)
-    if (cs.groups[g_begin + gi].nslots > 0) os << "    case " << gi << ": rx_fix_" << gi << "(p, acc); break;\n";
+    if (cs.groups[g_begin + gi].nslots > 0) os << "    case " << gi << ": rx_fix_" << gi << "(p, acc, sst); break;\n";
   os << "    default: break;\n  }\n}\n";
   return os.str();
 }

@@ -216,6 +216,49 @@ template <int K> DEV void rx_load_window(const RxParams &p, Ctx<K> &c, u32 (&pl)
   }
 }
 
+// split prologue (software pipelining): rx_fetch issues the 128-bit loads of
+// a window into registers, rx_unpack transposes them one window later
+template <int K> DEV void rx_fetch(const RxParams &p, u32 lane, u32 (&x)[K][8], i64 fword) {
+#pragma unroll
+  for (int i = 0; i < K; ++i) {
+    const i64 pos = (fword + (i64)(lane * K + i)) * 32;
+    if (p.aligned && pos >= p.avail_lo && pos + 32 <= p.avail_hi) {
+      const uint4 *q = reinterpret_cast<const uint4 *>(p.in + pos);
+      const uint4 a = __ldg(q), b = __ldg(q + 1);
+      x[i][0] = a.x; x[i][1] = a.y; x[i][2] = a.z; x[i][3] = a.w;
+      x[i][4] = b.x; x[i][5] = b.y; x[i][6] = b.z; x[i][7] = b.w;
+    } else {
+#pragma unroll
+      for (int j = 0; j < 8; ++j) x[i][j] = 0u;
+      for (int j = 0; j < 32; ++j) {
+        const i64 ps = pos + j;
+        if (ps >= p.avail_lo && ps < p.avail_hi) x[i][j >> 2] |= (u32)p.in[ps] << (8 * (j & 3));
+      }
+    }
+  }
+}
+
+template <int K> DEV void rx_unpack(const RxParams &p, Ctx<K> &c, const u32 (&x)[K][8], u32 (&pl)[8][K], i64 fword) {
+#pragma unroll
+  for (int i = 0; i < K; ++i) {
+    const i64 pos = (fword + (i64)(c.lane * K + i)) * 32;
+    u32 t[8];
+    rx_transpose32(x[i], t);
+#pragma unroll
+    for (int k = 0; k < 8; ++k) pl[k][i] = t[k];
+    const i64 lo = p.valid_lo - pos, hi = p.valid_hi - pos;
+    u32 m;
+    if (lo <= 0 && hi >= 32) m = RX_FULL;
+    else if (hi <= 0 || lo >= 32) m = 0u;
+    else {
+      const u32 a = lo <= 0 ? RX_FULL : (RX_FULL << (u32)lo);
+      const u32 b = hi >= 32 ? RX_FULL : (RX_FULL >> (u32)(32 - hi));
+      m = a & b;
+    }
+    c.vm[i] = m;
+  }
+}
+
 // committed mask: local words [Lw, Lw+cw), positions [0, len)
 template <int K> DEV void rx_commit_mask(const RxParams &p, Ctx<K> &c, int Lw, i64 fword) {
 #pragma unroll
@@ -260,120 +303,133 @@ template <class G> DEV void rx_ctx_init(const RxParams &p, Ctx<G::K> &c, u64 *ac
   __syncwarp();
 }
 
+// Per-warp state scratch in shared memory (warp-private; every lane reads
+// and writes the same uniform words): the body reads st[] (state carried in
+// from the previous window) and accumulates nst[] (state for the next one).
+DEV void rx_state_zero(u32 *a, int n, u32 lane) {
+  for (int s = (int)lane; s < n; s += 32) a[s] = 0u;
+  __syncwarp();
+}
+DEV void rx_state_copy(u32 *d, const u32 *s, int n, u32 lane) {
+  for (int i = (int)lane; i < n; i += 32) d[i] = s[i];
+  __syncwarp();
+}
+DEV bool rx_state_eq(const u32 *a, const u32 *b, int n, u32 lane) {
+  bool e = true;
+  for (int s = (int)lane; s < n; s += 32) e = e && (a[s] == b[s]);
+  return __all_sync(RX_FULL, e);
+}
+
 // Runs one group (traits G) over one segment (pass 1).
 template <class G>
-DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc) {
-  constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS > 0 ? G::NS : 1;
+DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst) {
+  constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS;
   const i64 len_words = rx_div_up(p.len, 32);
   const i64 nwin = rx_div_up(len_words, Bw);
   const i64 w_begin = (i64)seg * p.sw;
-  if (w_begin >= nwin && seg != 0) return;
-  const i64 w_end = w_begin + p.sw < nwin ? w_begin + p.sw : nwin;
+  const bool live = w_begin < nwin || seg == 0;
+  const i64 w_end = !live ? w_begin : (w_begin + p.sw < nwin ? w_begin + p.sw : nwin);
   Ctx<K> c;
   rx_ctx_init<G>(p, c, acc);
   u32 pl[8][K];
-  u32 st[NS], nst[NS];
-#pragma unroll
-  for (int s = 0; s < NS; ++s) st[s] = (seg == 0 && p.st_in) ? p.st_in[G::SBASE + s] : 0u;
-  for (i64 w = w_begin; w < w_end; ++w) {
-    const i64 cstart = w * Bw;
-    const i64 fword = cstart - Lw;
-    c.cw = (u32)((len_words - cstart) < Bw ? (len_words - cstart) : Bw);
-    c.word0 = fword;
-    rx_load_window(p, c, pl, fword);
-    rx_commit_mask(p, c, Lw, fword);
-#pragma unroll
-    for (int s = 0; s < NS; ++s) nst[s] = 0u;
-    G::body(c, pl, st, nst);
-#pragma unroll
-    for (int s = 0; s < NS; ++s) st[s] = nst[s];
+  u32 xr[K][8];
+  u32 *st = sst, *nst = sst + G::NSMAX;
+  for (int s = (int)c.lane; s < NS; s += 32) st[s] = (seg == 0 && p.st_in) ? p.st_in[G::SBASE + s] : 0u;
+  __syncwarp();
+  if (w_begin < w_end) rx_fetch<K>(p, c.lane, xr, w_begin * Bw - Lw);
+  // All warps of the CTA run this group; they step through their windows in
+  // lockstep (one barrier per window) so that the SM fetches each line of
+  // the group's straight-line program once for all of them.
+  for (int i = 0; i < p.sw; ++i) {
+    const i64 w = w_begin + i;
+    if (w < w_end) {
+      const i64 cstart = w * Bw;
+      const i64 fword = cstart - Lw;
+      c.cw = (u32)((len_words - cstart) < Bw ? (len_words - cstart) : Bw);
+      c.word0 = fword;
+      rx_unpack<K>(p, c, xr, pl, fword);
+      if (w + 1 < w_end) rx_fetch<K>(p, c.lane, xr, fword + Bw);  // prefetch the next window
+      rx_commit_mask(p, c, Lw, fword);
+      if (NS > 0) rx_state_zero(nst, NS, c.lane);
+      G::body(c, pl, st, nst);
+      u32 *t = st;
+      st = nst;
+      nst = t;
+      __syncwarp();
+    }
+    __syncthreads();
   }
-  if (G::NS > 0) {
+  if (!live) return;
+  if (NS > 0) {
     u32 *dst = p.seg_state + ((i64)seg * G::NG + G::GID) * G::NSMAX;
-    if (c.lane == 0) {
-#pragma unroll
-      for (int s = 0; s < NS; ++s) dst[s] = st[s];
-    }
-    if (p.st_out && w_end == nwin && c.lane == 0) {
-#pragma unroll
-      for (int s = 0; s < NS; ++s) p.st_out[G::SBASE + s] = st[s];
-    }
+    for (int s = (int)c.lane; s < NS; s += 32) dst[s] = st[s];
+    if (p.st_out && w_end == nwin)
+      for (int s = (int)c.lane; s < NS; s += 32) p.st_out[G::SBASE + s] = st[s];
   }
   rx_flush<G>(p, c);
-}
-
-template <int NS> DEV bool rx_state_eq(const u32 *a, const u32 *b) {
-  bool e = true;
-#pragma unroll
-  for (int s = 0; s < NS; ++s) e = e && (a[s] == b[s]);
-  return e;
 }
 
 // Fix-up / rematch (one warp per group): walk the windows in order carrying
 // the true state; wherever it differs from the state pass 1 used, re-run the
 // window with both states and apply (new - old) until they agree.
 template <class G>
-DEV void rx_fixup_group(const RxParams &p, u64 *acc) {
-  constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS > 0 ? G::NS : 1;
-  if (G::NS == 0) return;
+DEV void rx_fixup_group(const RxParams &p, u64 *acc, u32 *sst) {
+  constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS, M = G::NSMAX;
+  if (NS == 0) return;
   const i64 len_words = rx_div_up(p.len, 32);
   const i64 nwin = rx_div_up(len_words, Bw);
   const i64 nseg = rx_div_up(nwin, p.sw);
   Ctx<K> c;
   rx_ctx_init<G>(p, c, acc);
   u32 pl[8][K];
-  u32 tru[NS], old[NS], t1[NS], t2[NS];
-#pragma unroll
-  for (int s = 0; s < NS; ++s) {
+  u32 xr[K][8];
+  u32 *tru = sst, *old = sst + M, *t1 = sst + 2 * M, *t2 = sst + 3 * M;
+  for (int s = (int)c.lane; s < NS; s += 32) {
     tru[s] = p.st_in ? p.st_in[G::SBASE + s] : 0u;
     old[s] = (p.mode == 2 && p.st_assumed) ? p.st_assumed[G::SBASE + s] : 0u;
   }
+  __syncwarp();
   for (i64 seg = 0; seg < nseg; ++seg) {
     const i64 w_begin = seg * p.sw;
     const i64 w_end = w_begin + p.sw < nwin ? w_begin + p.sw : nwin;
     if (p.mode == 1) {
       // the state pass 1 assumed for this segment
-#pragma unroll
-      for (int s = 0; s < NS; ++s) old[s] = seg == 0 ? (p.st_in ? p.st_in[G::SBASE + s] : 0u) : 0u;
+      for (int s = (int)c.lane; s < NS; s += 32) old[s] = seg == 0 ? (p.st_in ? p.st_in[G::SBASE + s] : 0u) : 0u;
+      __syncwarp();
     }
-    bool conv = rx_state_eq<NS>(tru, old);
+    bool conv = rx_state_eq(tru, old, NS, c.lane);
     for (i64 w = w_begin; w < w_end && !conv; ++w) {
       const i64 cstart = w * Bw;
       const i64 fword = cstart - Lw;
       c.cw = (u32)((len_words - cstart) < Bw ? (len_words - cstart) : Bw);
       c.word0 = fword;
-      rx_load_window(p, c, pl, fword);
+      rx_fetch<K>(p, c.lane, xr, fword);
+      rx_unpack<K>(p, c, xr, pl, fword);
       rx_commit_mask(p, c, Lw, fword);
       // old run: subtract
       c.sign = ~0ull;
       c.want_dense = false;
-#pragma unroll
-      for (int s = 0; s < NS; ++s) t1[s] = 0u;
+      rx_state_zero(t1, NS, c.lane);
       G::body(c, pl, old, t1);
       // new run: add, rewrite dense words
       c.sign = 1ull;
       c.want_dense = p.dense != nullptr;
-#pragma unroll
-      for (int s = 0; s < NS; ++s) t2[s] = 0u;
+      rx_state_zero(t2, NS, c.lane);
       G::body(c, pl, tru, t2);
-#pragma unroll
-      for (int s = 0; s < NS; ++s) {
-        old[s] = t1[s];
-        tru[s] = t2[s];
-      }
-      conv = rx_state_eq<NS>(tru, old);
+      __syncwarp();
+      rx_state_copy(old, t1, NS, c.lane);
+      rx_state_copy(tru, t2, NS, c.lane);
+      conv = rx_state_eq(tru, old, NS, c.lane);
     }
     if (conv) {
       if (p.mode == 2) break;  // identical to the caller's run from here on
       // from here on pass 1's result stands: take its segment end state
       const u32 *src = p.seg_state + (seg * G::NG + G::GID) * G::NSMAX;
-#pragma unroll
-      for (int s = 0; s < NS; ++s) tru[s] = src[s];
+      for (int s = (int)c.lane; s < NS; s += 32) tru[s] = src[s];
+      __syncwarp();
     }
-    if (seg == nseg - 1 && p.st_out && c.lane == 0 && (p.mode == 1 || !conv)) {
-#pragma unroll
-      for (int s = 0; s < NS; ++s) p.st_out[G::SBASE + s] = tru[s];
-    }
+    if (seg == nseg - 1 && p.st_out && (p.mode == 1 || !conv))
+      for (int s = (int)c.lane; s < NS; s += 32) p.st_out[G::SBASE + s] = tru[s];
   }
   rx_flush<G>(p, c);
 }

@@ -197,14 +197,16 @@ struct Lowerer {
 
   // Concatenation items[j..] after a prefix whose (possibly empty) end
   // markers are P and whose non-empty end markers are N.
-  int E_cat(const std::vector<Item> &items, size_t j, int P, int N) {
+  int E_cat(const std::vector<Item> &items, size_t j, int P, int N, bool guarded = false) {
     for (; j < items.size(); ++j) {
       // Zero-block-skipping guard (Sec. 6): P is a zero-path
       // head -- if P is all-zero in a window, everything downstream in this
-      // concatenation (and N, a subset of P) is zero.  First guard after the
-      // first shift+AND, then every `interval` instructions.
+      // concatenation (and N, a subset of P) is zero.  First guard at the
+      // head of the path (after its first shift+AND), then every `interval`
+      // instructions.
+      const bool head = !guarded && ir.nodes[P].op == Op::And;
       if (opt.interval > 0 && loops.empty() && j > 0 && !is(P, Op::Ones) && !is(P, Op::Zero) &&
-          since_guard >= (size_t)opt.interval && ir.nodes[P].op != Op::CC) {
+          (head || since_guard >= (size_t)opt.interval) && ir.nodes[P].op != Op::CC) {
         Node g;
         g.op = Op::Guard;
         g.a = P;
@@ -212,7 +214,7 @@ struct Lowerer {
         ir.n_guards++;
         int sb = push_block();
         since_guard = 0;
-        int res = E_cat(items, j, P, N);
+        int res = E_cat(items, j, P, N, true);
         pop_block();
         ir.nodes[gid].sub = sb;
         ir.nodes[gid].res = res;
@@ -229,7 +231,6 @@ struct Lowerer {
         P = e;
         N = e;
       }
-      if (j == 0 && ir.n_guards == 0) since_guard = std::max<size_t>(since_guard, 0);
       if (is(P, Op::Zero)) return zero;
     }
     return N;
@@ -464,9 +465,9 @@ bool plan_groups(CompiledSet &cs, int group_size, int force_K, std::string &why)
   for (auto &r : cs.irs) total_instr += r.n_instr;
   if (group_size <= 0) {
     // aim for <= ~64 regexes and a bounded code size per group
-    group_size = 16;
+    group_size = 32;
   }
-  const size_t max_instr = 600;
+  const size_t max_instr = 1500;  // bounds one NVRTC unit (compile time) and the group's code size
   cs.groups.clear();
   Group g;
   size_t gi = 0;

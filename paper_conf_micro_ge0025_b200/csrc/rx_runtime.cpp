@@ -413,18 +413,20 @@ rx_status ensure_loaded(rx_program *p, int &device) {
   return RX_OK;
 }
 
-constexpr int kWarpsPerBlock = 4;
+constexpr int kPass1Warps = 16;  // one CTA = one SM's worth of warps, one group (lockstep)
+constexpr int kFixupWarps = 4;
 
-rx_status launch(RxModule &m, CUfunction f, long long warps, const RxParamsHost &prm, cudaStream_t s) {
+rx_status launch(RxModule &m, CUfunction f, long long blocks, int warps_per_block, const RxParamsHost &prm,
+                 cudaStream_t s) {
   Drv &d = drv();
-  if (warps <= 0) return RX_OK;
-  long long blocks = (warps + kWarpsPerBlock - 1) / kWarpsPerBlock;
+  if (blocks <= 0) return RX_OK;
   if (blocks > 0x7fffffffLL) return fail(RX_EINVAL, "grid too large");
-  unsigned smem = (unsigned)(kWarpsPerBlock * 3 * m.nr_max * sizeof(unsigned long long));
+  unsigned smem = (unsigned)(warps_per_block * (3 * m.nr_max * sizeof(unsigned long long) + 4 * m.ns_max * 4));
   if (smem > 48 * 1024) d.FuncSetAttribute(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)smem);
   RxParamsHost local = prm;
   void *args[] = {&local};
-  CUresult r = d.LaunchKernel(f, (unsigned)blocks, 1, 1, 32 * kWarpsPerBlock, 1, 1, smem, (CUstream)s, args, nullptr);
+  CUresult r =
+      d.LaunchKernel(f, (unsigned)blocks, 1, 1, 32 * warps_per_block, 1, 1, smem, (CUstream)s, args, nullptr);
   if (r != CUDA_SUCCESS) return fail(RX_ECUDA, "cuLaunchKernel failed: " + std::to_string((int)r));
   return RX_OK;
 }
@@ -490,7 +492,7 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
     for (auto &m : p->mods) {
       if (!m.any_state) continue;
       prm.seg_state = nullptr;
-      s = launch(m, m.fixup, m.g_end - m.g_begin, prm, stream);
+      s = launch(m, m.fixup, div_up(m.g_end - m.g_begin, kFixupWarps), kFixupWarps, prm, stream);
       if (s != RX_OK) return s;
     }
     if (status_scratch) cudaFreeAsync(status_scratch, stream);
@@ -499,9 +501,12 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
   // segments: enough warps to fill the GPU several times over
   long long max_nwin = 0;
   for (auto &g : p->cs.groups) max_nwin = std::max(max_nwin, div_up(len_words, g.Bw));
-  const long long target_warps = 148LL * 16 * 4;
-  long long sw = std::max<long long>(4, div_up(max_nwin * G, target_warps));
+  // pass-1 CTAs: 16 segments of one group each; aim for ~4 waves of 148 SMs
+  const long long target_ctas = 148LL * 4;
+  const long long cpg0 = std::max<long long>(1, div_up(target_ctas, std::max(G, 1)));
+  long long sw = std::max<long long>(4, div_up(max_nwin, cpg0 * kPass1Warps));
   long long nseg_max = std::max<long long>(1, div_up(max_nwin, sw));
+  const long long cpg = div_up(nseg_max, kPass1Warps);
   prm.sw = (int)std::min<long long>(sw, 1 << 30);
   prm.nseg_max = (int)nseg_max;
   prm.mode = 0;
@@ -514,11 +519,11 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
     }
     prm.seg_state = seg_state;
     prm.mode = 0;
-    s = launch(m, m.pass1, nseg_max * mg, prm, stream);
+    s = launch(m, m.pass1, cpg * mg, kPass1Warps, prm, stream);
     if (s != RX_OK) return s;
     if (m.any_state) {
       prm.mode = 1;
-      s = launch(m, m.fixup, mg, prm, stream);
+      s = launch(m, m.fixup, div_up(mg, kFixupWarps), kFixupWarps, prm, stream);
       if (s != RX_OK) return s;
       cudaFreeAsync(seg_state, stream);
     }
