@@ -68,7 +68,9 @@ typedef struct {
   uint32_t reserved[3];
 } rx_options;
 
-#define RX_F_NO_REBALANCE 1u /* disable Shift Rebalancing (Sec. 5) */
+#define RX_F_NO_REBALANCE 1u /* force Shift Rebalancing off */
+#define RX_F_REBALANCE 8u    /* enable Shift Rebalancing (Sec. 5); off by default: on B200 it buys
+                                ILP only (no shift barriers at warp scope) -- see DESIGN.md */
 #define RX_F_NO_GUARDS 2u    /* disable Zero Block Skipping (Sec. 6) */
 #define RX_F_NO_CACHE 4u     /* do not read/write the on-disk cubin cache */
 

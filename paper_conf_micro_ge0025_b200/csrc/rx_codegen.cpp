@@ -38,12 +38,16 @@ struct RegexEmitter {
   int K;
   int rloc;       // member index in the group
   int slot_base;  // first state slot of this regex in the group
-  std::vector<std::map<TabKey, std::string>> cc_scope;
-  std::vector<std::map<std::vector<uint64_t>, std::string>> set_scope;
+  // CC / BDD-node caches by scope; scope 0 is shared by all regexes of the
+  // group (their unguarded heads), deeper scopes are guard / loop bodies
+  std::vector<std::map<TabKey, std::string>> &cc_scope;
+  std::vector<std::map<std::vector<uint64_t>, std::string>> &set_scope;
   int tmp = 0;
 
-  RegexEmitter(std::ostringstream &o, const RegexIR &r, int k, int rl, int sb)
-      : os(o), ir(r), K(k), rloc(rl), slot_base(sb) {}
+  RegexEmitter(std::ostringstream &o, const RegexIR &r, int k, int rl, int sb,
+               std::vector<std::map<TabKey, std::string>> &ccs,
+               std::vector<std::map<std::vector<uint64_t>, std::string>> &sets)
+      : os(o), ir(r), K(k), rloc(rl), slot_base(sb), cc_scope(ccs), set_scope(sets) {}
 
   std::string ind(int n) { return std::string(2 * n, ' '); }
   std::string nv(int id) { return "n" + std::to_string(rloc) + "_" + std::to_string(id); }
@@ -335,10 +339,8 @@ struct RegexEmitter {
   }
 
   void emit_regex() {
-    os << "    {  // regex member " << rloc << "\n";
-    push();
+    os << "    // ---- regex member " << rloc << " (unguarded classes shared with the group)\n";
     block(0, 3, "");
-    pop();
     const Node &o = ir.nodes[ir.out];
     if (o.op != Op::Zero) {
       std::string R = nv(ir.out);
@@ -350,7 +352,6 @@ struct RegexEmitter {
       os << "        rx_emit<" << K << ">(c, " << rloc << ", ov);\n";
       os << "      }\n";
     }
-    os << "    }\n";
   }
 };
 
@@ -397,16 +398,31 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
     for (int k = 0; k < 8; ++k)
       for (int i = 0; i < g.K; ++i) os << "    const u32 b" << k << "w" << i << " = pl[" << k << "][" << i << "];\n";
     for (int i = 0; i < g.K; ++i) os << "    const u32 vmw" << i << " = c.vm[" << i << "];\n";
+    std::vector<std::map<TabKey, std::string>> ccs(1);
+    std::vector<std::map<std::vector<uint64_t>, std::string>> sets(1);
     for (size_t m = 0; m < g.regexes.size(); ++m) {
-      RegexEmitter em(os, cs.irs[g.regexes[m]], g.K, (int)m, g.slot_base[m]);
+      RegexEmitter em(os, cs.irs[g.regexes[m]], g.K, (int)m, g.slot_base[m], ccs, sets);
       em.emit_regex();
     }
     os << "  }\n};\n";
     os << "extern \"C\" __device__ __noinline__ void rx_seg_" << gi
-       << "(const RxParams &p, int seg, u64 *acc, u32 *sst) { rx_run_segment<RxG" << gi << ">(p, seg, acc, sst); }\n";
+       << "(const RxParams &p, int seg) {\n"
+       // shared memory: [wpb][3*NRMAX] u64 accumulators | [wpb][4*NSMAX] u32 state |
+       // [wpb][2][2048] window staging (TMA) | [wpb][2] u64 mbarriers
+       << "  extern __shared__ __align__(16) u64 rx_smem[];\n"
+       << "  const int warp = threadIdx.x >> 5, wpb = blockDim.x >> 5;\n"
+       << "  u64 *acc = rx_smem + warp * (3 * " << nrmax << ");\n"
+       << "  u32 *st0 = reinterpret_cast<u32 *>(rx_smem + wpb * (3 * " << nrmax << "));\n"
+       << "  unsigned char *tb0 = reinterpret_cast<unsigned char *>(st0 + ((wpb * (4 * " << nsmax
+       << ") + 3) & ~3));\n"
+       << "  u64 *bars = reinterpret_cast<u64 *>(tb0 + wpb * 4096) + 2 * warp;\n"
+       << "  rx_run_segment<RxG" << gi << ">(p, seg, acc, st0 + warp * (4 * " << nsmax << "), tb0 + warp * 4096, bars);\n}\n";
     if (g.nslots > 0)
-      os << "extern \"C\" __device__ __noinline__ void rx_fix_" << gi
-         << "(const RxParams &p, u64 *acc, u32 *sst) { rx_fixup_group<RxG" << gi << ">(p, acc, sst); }\n";
+      os << "extern \"C\" __device__ __noinline__ void rx_fix_" << gi << "(const RxParams &p) {\n"
+         << "  extern __shared__ u64 rx_smem[];\n"
+         << "  const int warp = threadIdx.x >> 5, wpb = blockDim.x >> 5;\n"
+         << "  rx_fixup_group<RxG" << gi << ">(p, rx_smem + warp * (3 * " << nrmax << "),\n"
+         << "      reinterpret_cast<u32 *>(rx_smem + wpb * (3 * " << nrmax << ")) + warp * (4 * " << nsmax << "));\n}\n";
   }
   return os.str();
 }
@@ -422,39 +438,31 @@ std::string emit_kernel_unit(CompiledSet &cs) {
   int G = (int)cs.groups.size();
   os << "#define RX_NG " << G << "\n#define RX_NSMAX " << nsmax << "\n#define RX_NRMAX " << nrmax << "\n";
   for (int gi = 0; gi < G; ++gi) {
-    os << "extern \"C\" __device__ void rx_seg_" << gi << "(const RxParams &p, int seg, u64 *acc, u32 *sst);\n";
-    if (cs.groups[gi].nslots > 0)
-      os << "extern \"C\" __device__ void rx_fix_" << gi << "(const RxParams &p, u64 *acc, u32 *sst);\n";
+    os << "extern \"C\" __device__ void rx_seg_" << gi << "(const RxParams &p, int seg);\n";
+    if (cs.groups[gi].nslots > 0) os << "extern \"C\" __device__ void rx_fix_" << gi << "(const RxParams &p);\n";
   }
   int g_begin = 0;
   // pass 1: one CTA of 16 warps (the whole SM's register file) runs one
   // group over 16 consecutive segments in lockstep, so the SM's instruction
   // caches hold one program at a time
   os << "\nextern \"C\" __global__ void __launch_bounds__(512, 1) rx_pass1(const RxParams p) {\n"
-        "  extern __shared__ u64 rx_smem[];\n"
         "  const int warp = threadIdx.x >> 5;\n"
         "  const int wpb = blockDim.x >> 5;\n"
-        // shared memory per warp: [3*NRMAX] u64 accumulators, then [4*NSMAX] u32 state
-        "  u64 *acc = rx_smem + warp * (3 * RX_NRMAX);\n"
-        "  u32 *sst = reinterpret_cast<u32 *>(rx_smem + wpb * (3 * RX_NRMAX)) + warp * (4 * RX_NSMAX);\n"
         "  const int cpg = (p.nseg_max + wpb - 1) / wpb;  // CTAs per group\n"
         "  const int g = (int)(blockIdx.x / cpg);\n"
         "  const long long seg = (long long)(blockIdx.x % cpg) * wpb + warp;\n"
         "  if (g >= RX_NG) return;\n"
         "  switch (g) {\n";
-  for (int gi = 0; gi < G; ++gi) os << "    case " << gi << ": rx_seg_" << gi << "(p, (int)seg, acc, sst); break;\n";
+  for (int gi = 0; gi < G; ++gi) os << "    case " << gi << ": rx_seg_" << gi << "(p, (int)seg); break;\n";
   os << "    default: break;\n  }\n}\n";
   os << "\nextern \"C\" __global__ void __launch_bounds__(128) rx_fixup(const RxParams p) {\n"
-        "  extern __shared__ u64 rx_smem[];\n"
         "  const int warp = threadIdx.x >> 5;\n"
         "  const int wpb = blockDim.x >> 5;\n"
-        "  u64 *acc = rx_smem + warp * (3 * RX_NRMAX);\n"
-        "  u32 *sst = reinterpret_cast<u32 *>(rx_smem + wpb * (3 * RX_NRMAX)) + warp * (4 * RX_NSMAX);\n"
         "  const long long g = (long long)blockIdx.x * wpb + warp;\n"
         "  if (g >= RX_NG) return;\n"
         "  switch ((int)g) {\n";
   for (int gi = 0; gi < G; ++gi)
-    if (cs.groups[g_begin + gi].nslots > 0) os << "    case " << gi << ": rx_fix_" << gi << "(p, acc, sst); break;\n";
+    if (cs.groups[g_begin + gi].nslots > 0) os << "    case " << gi << ": rx_fix_" << gi << "(p); break;\n";
   os << "    default: break;\n  }\n}\n";
   return os.str();
 }

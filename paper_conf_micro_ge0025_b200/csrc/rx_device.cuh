@@ -217,57 +217,88 @@ template <int K> DEV void rx_load_window(const RxParams &p, Ctx<K> &c, u32 (&pl)
 }
 
 // split prologue (software pipelining): rx_fetch issues the 128-bit loads of
-// a window into registers, rx_unpack transposes them one window later
-template <int K> DEV void rx_fetch(const RxParams &p, u32 lane, u32 (&x)[K][8], i64 fword) {
+// a window into registers, rx_unpack transposes them one window later.
+// Interior windows (all bytes readable and valid, 16-byte aligned) take the
+// straight path; edge windows go through an out-of-line byte loader.
+struct RxW8 {
+  u32 v[8];
+};
+static __device__ __noinline__ RxW8 rx_fetch_word_slow(const unsigned char *in, i64 avail_lo, i64 avail_hi, i64 pos) {
+  RxW8 r;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) r.v[j] = 0u;
+  for (int j = 0; j < 32; ++j) {
+    const i64 ps = pos + j;
+    if (ps >= avail_lo && ps < avail_hi) r.v[j >> 2] |= (u32)in[ps] << (8 * (j & 3));
+  }
+  return r;
+}
+
+struct RxRange {  // words of the chunk whose windows need no edge handling
+  i64 lo, hi;     // a frame [fword, fword+32K) is interior iff lo <= fword && fword+32K <= hi
+  i64 len_words_full;  // words entirely below len
+};
+DEV RxRange rx_interior(const RxParams &p) {
+  RxRange r;
+  const i64 lo = p.avail_lo > p.valid_lo ? p.avail_lo : p.valid_lo;
+  const i64 hi = p.avail_hi < p.valid_hi ? p.avail_hi : p.valid_hi;
+  r.lo = p.aligned ? (lo + 31 >= 0 ? (lo + 31) / 32 : -((-(lo + 31) + 31) / 32)) : ((i64)1 << 62);
+  r.hi = p.aligned ? (hi >= 0 ? hi / 32 : -((-hi + 31) / 32)) : -((i64)1 << 62);
+  r.len_words_full = p.len / 32;
+  return r;
+}
+
+template <int K> DEV void rx_fetch(const RxParams &p, const RxRange &ir, u32 lane, u32 (&x)[K][8], i64 fword) {
+  const bool interior = fword >= ir.lo && fword + 32 * K <= ir.hi;
 #pragma unroll
   for (int i = 0; i < K; ++i) {
     const i64 pos = (fword + (i64)(lane * K + i)) * 32;
-    if (p.aligned && pos >= p.avail_lo && pos + 32 <= p.avail_hi) {
+    if (interior) {
       const uint4 *q = reinterpret_cast<const uint4 *>(p.in + pos);
       const uint4 a = __ldg(q), b = __ldg(q + 1);
       x[i][0] = a.x; x[i][1] = a.y; x[i][2] = a.z; x[i][3] = a.w;
       x[i][4] = b.x; x[i][5] = b.y; x[i][6] = b.z; x[i][7] = b.w;
     } else {
+      const RxW8 r = rx_fetch_word_slow(p.in, p.avail_lo, p.avail_hi, pos);
 #pragma unroll
-      for (int j = 0; j < 8; ++j) x[i][j] = 0u;
-      for (int j = 0; j < 32; ++j) {
-        const i64 ps = pos + j;
-        if (ps >= p.avail_lo && ps < p.avail_hi) x[i][j >> 2] |= (u32)p.in[ps] << (8 * (j & 3));
-      }
+      for (int j = 0; j < 8; ++j) x[i][j] = r.v[j];
     }
   }
 }
 
-template <int K> DEV void rx_unpack(const RxParams &p, Ctx<K> &c, const u32 (&x)[K][8], u32 (&pl)[8][K], i64 fword) {
+template <int K>
+DEV void rx_unpack(const RxParams &p, const RxRange &ir, Ctx<K> &c, const u32 (&x)[K][8], u32 (&pl)[8][K], i64 fword) {
+  const bool interior = fword >= ir.lo && fword + 32 * K <= ir.hi;
 #pragma unroll
   for (int i = 0; i < K; ++i) {
-    const i64 pos = (fword + (i64)(c.lane * K + i)) * 32;
     u32 t[8];
     rx_transpose32(x[i], t);
 #pragma unroll
     for (int k = 0; k < 8; ++k) pl[k][i] = t[k];
-    const i64 lo = p.valid_lo - pos, hi = p.valid_hi - pos;
-    u32 m;
-    if (lo <= 0 && hi >= 32) m = RX_FULL;
-    else if (hi <= 0 || lo >= 32) m = 0u;
-    else {
-      const u32 a = lo <= 0 ? RX_FULL : (RX_FULL << (u32)lo);
-      const u32 b = hi >= 32 ? RX_FULL : (RX_FULL >> (u32)(32 - hi));
-      m = a & b;
+    u32 m = RX_FULL;
+    if (!interior) {
+      const i64 pos = (fword + (i64)(c.lane * K + i)) * 32;
+      const i64 lo = p.valid_lo - pos, hi = p.valid_hi - pos;
+      if (hi <= 0 || lo >= 32) m = 0u;
+      else if (!(lo <= 0 && hi >= 32)) {
+        const u32 a = lo <= 0 ? RX_FULL : (RX_FULL << (u32)lo);
+        const u32 b = hi >= 32 ? RX_FULL : (RX_FULL >> (u32)(32 - hi));
+        m = a & b;
+      }
     }
     c.vm[i] = m;
   }
 }
 
 // committed mask: local words [Lw, Lw+cw), positions [0, len)
-template <int K> DEV void rx_commit_mask(const RxParams &p, Ctx<K> &c, int Lw, i64 fword) {
+template <int K> DEV void rx_commit_mask(const RxParams &p, const RxRange &ir, Ctx<K> &c, int Lw, i64 fword) {
+  const bool full = fword + Lw + (i64)c.cw <= ir.len_words_full;
 #pragma unroll
   for (int i = 0; i < K; ++i) {
     const int j = (int)(c.lane * K + i);
-    u32 m = 0u;
-    if (j >= Lw && j < Lw + (int)c.cw) {
-      const i64 pos = (fword + j) * 32;
-      const i64 hi = p.len - pos;
+    u32 m = (j >= Lw && j < Lw + (int)c.cw) ? RX_FULL : 0u;
+    if (!full && m) {
+      const i64 hi = p.len - (fword + j) * 32;
       m = hi >= 32 ? RX_FULL : (hi <= 0 ? 0u : (RX_FULL >> (u32)(32 - hi)));
     }
     c.cm[i] = m;
@@ -320,10 +351,124 @@ DEV bool rx_state_eq(const u32 *a, const u32 *b, int n, u32 lane) {
   return __all_sync(RX_FULL, e);
 }
 
-// Runs one group (traits G) over one segment (pass 1).
+// ---------------------------------------------------------------------------
+// TMA (bulk async copy) staging of window bytes: one elected lane copies the
+// next window's 1024*K contiguous bytes global -> shared memory, completion
+// tracked by an mbarrier (transaction bytes); double-buffered per warp.
+// ---------------------------------------------------------------------------
+DEV u32 rx_smem_addr(const void *p) { return (u32)__cvta_generic_to_shared(p); }
+DEV void rx_mbar_init(u64 *bar, u32 count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(rx_smem_addr(bar)), "r"(count) : "memory");
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+DEV void rx_bulk_load(void *dst, const void *src, u32 bytes, u64 *bar) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(rx_smem_addr(bar)), "r"(bytes)
+               : "memory");
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   rx_smem_addr(dst)),
+               "l"(src), "r"(bytes), "r"(rx_smem_addr(bar))
+               : "memory");
+}
+DEV void rx_mbar_wait(u64 *bar, u32 phase) {
+  u32 done = 0;
+  while (!done) {
+    asm volatile(
+        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+        : "=r"(done)
+        : "r"(rx_smem_addr(bar)), "r"(phase)
+        : "memory");
+  }
+}
+
+// Runs one group (traits G) over one segment (pass 1).  Windows of groups
+// with K <= 2 are staged through shared memory by TMA bulk copies issued
+// one window ahead; wider groups prefetch into registers.
 template <class G>
-DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst) {
+DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *tbuf, u64 *bars) {
   constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS;
+  constexpr u32 WB = 1024u * K;  // window bytes
+  if constexpr (K <= 2) {
+    const i64 len_words = rx_div_up(p.len, 32);
+    const i64 nwin = rx_div_up(len_words, Bw);
+    const i64 w_begin = (i64)seg * p.sw;
+    const bool live = w_begin < nwin || seg == 0;
+    const i64 w_end = !live ? w_begin : (w_begin + p.sw < nwin ? w_begin + p.sw : nwin);
+    Ctx<K> c;
+    rx_ctx_init<G>(p, c, acc);
+    u32 pl[8][K];
+    u32 xr[K][8];
+    u32 *st = sst, *nst = sst + G::NSMAX;
+    for (int s = (int)c.lane; s < NS; s += 32) st[s] = (seg == 0 && p.st_in) ? p.st_in[G::SBASE + s] : 0u;
+    if (c.lane == 0) {
+      rx_mbar_init(&bars[0], 1);
+      rx_mbar_init(&bars[1], 1);
+    }
+    __syncwarp();
+    const RxRange ir = rx_interior(p);
+    bool issued0 = false, issued1 = false;
+    u32 ph0 = 0, ph1 = 0;
+    if (w_begin < w_end) {
+      const i64 f0 = w_begin * Bw - Lw;
+      if (f0 >= ir.lo && f0 + 32 * K <= ir.hi) {
+        if (c.lane == 0) rx_bulk_load(tbuf, p.in + f0 * 32, WB, &bars[0]);
+        issued0 = true;
+      }
+    }
+    for (int i = 0; i < p.sw; ++i) {
+      const i64 w = w_begin + i;
+      const int b = i & 1;
+      if (w < w_end) {
+        const i64 cstart = w * Bw;
+        const i64 fword = cstart - Lw;
+        c.cw = (u32)((len_words - cstart) < Bw ? (len_words - cstart) : Bw);
+        c.word0 = fword;
+        const bool staged = b ? issued1 : issued0;
+        if (staged) {
+          rx_mbar_wait(&bars[b], b ? ph1 : ph0);
+          if (b) { ph1 ^= 1u; issued1 = false; } else { ph0 ^= 1u; issued0 = false; }
+          const uint4 *q = reinterpret_cast<const uint4 *>(tbuf + b * WB + c.lane * (32u * K));
+#pragma unroll
+          for (int k = 0; k < K; ++k) {
+            const uint4 a0 = q[2 * k], a1 = q[2 * k + 1];
+            xr[k][0] = a0.x; xr[k][1] = a0.y; xr[k][2] = a0.z; xr[k][3] = a0.w;
+            xr[k][4] = a1.x; xr[k][5] = a1.y; xr[k][6] = a1.z; xr[k][7] = a1.w;
+          }
+        } else {
+          rx_fetch<K>(p, ir, c.lane, xr, fword);
+        }
+        // stage the next window into the other buffer (read by every lane
+        // one window ago, released by the barrier that ended it)
+        if (w + 1 < w_end) {
+          const i64 nf = fword + Bw;
+          if (nf >= ir.lo && nf + 32 * K <= ir.hi) {
+            __syncwarp();
+            if (c.lane == 0) rx_bulk_load(tbuf + (b ^ 1) * WB, p.in + nf * 32, WB, &bars[b ^ 1]);
+            if (b) issued0 = true; else issued1 = true;
+          }
+        }
+        rx_unpack<K>(p, ir, c, xr, pl, fword);
+        rx_commit_mask(p, ir, c, Lw, fword);
+        if (NS > 0) rx_state_zero(nst, NS, c.lane);
+        G::body(c, pl, st, nst);
+        u32 *t = st;
+        st = nst;
+        nst = t;
+        __syncwarp();
+      }
+      __syncthreads();
+    }
+    if (!live) return;
+    if (NS > 0) {
+      u32 *dst = p.seg_state + ((i64)seg * G::NG + G::GID) * G::NSMAX;
+      for (int s = (int)c.lane; s < NS; s += 32) dst[s] = st[s];
+      if (p.st_out && w_end == nwin)
+        for (int s = (int)c.lane; s < NS; s += 32) p.st_out[G::SBASE + s] = st[s];
+    }
+    rx_flush<G>(p, c);
+    return;
+  }
+  (void)tbuf;
+  (void)bars;
   const i64 len_words = rx_div_up(p.len, 32);
   const i64 nwin = rx_div_up(len_words, Bw);
   const i64 w_begin = (i64)seg * p.sw;
@@ -336,7 +481,8 @@ DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst) {
   u32 *st = sst, *nst = sst + G::NSMAX;
   for (int s = (int)c.lane; s < NS; s += 32) st[s] = (seg == 0 && p.st_in) ? p.st_in[G::SBASE + s] : 0u;
   __syncwarp();
-  if (w_begin < w_end) rx_fetch<K>(p, c.lane, xr, w_begin * Bw - Lw);
+  const RxRange ir = rx_interior(p);
+  if (w_begin < w_end) rx_fetch<K>(p, ir, c.lane, xr, w_begin * Bw - Lw);
   // All warps of the CTA run this group; they step through their windows in
   // lockstep (one barrier per window) so that the SM fetches each line of
   // the group's straight-line program once for all of them.
@@ -347,9 +493,9 @@ DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst) {
       const i64 fword = cstart - Lw;
       c.cw = (u32)((len_words - cstart) < Bw ? (len_words - cstart) : Bw);
       c.word0 = fword;
-      rx_unpack<K>(p, c, xr, pl, fword);
-      if (w + 1 < w_end) rx_fetch<K>(p, c.lane, xr, fword + Bw);  // prefetch the next window
-      rx_commit_mask(p, c, Lw, fword);
+      rx_unpack<K>(p, ir, c, xr, pl, fword);
+      if (w + 1 < w_end) rx_fetch<K>(p, ir, c.lane, xr, fword + Bw);  // prefetch the next window
+      rx_commit_mask(p, ir, c, Lw, fword);
       if (NS > 0) rx_state_zero(nst, NS, c.lane);
       G::body(c, pl, st, nst);
       u32 *t = st;
@@ -403,9 +549,10 @@ DEV void rx_fixup_group(const RxParams &p, u64 *acc, u32 *sst) {
       const i64 fword = cstart - Lw;
       c.cw = (u32)((len_words - cstart) < Bw ? (len_words - cstart) : Bw);
       c.word0 = fword;
-      rx_fetch<K>(p, c.lane, xr, fword);
-      rx_unpack<K>(p, c, xr, pl, fword);
-      rx_commit_mask(p, c, Lw, fword);
+      const RxRange ir = rx_interior(p);
+      rx_fetch<K>(p, ir, c.lane, xr, fword);
+      rx_unpack<K>(p, ir, c, xr, pl, fword);
+      rx_commit_mask(p, ir, c, Lw, fword);
       // old run: subtract
       c.sign = ~0ull;
       c.want_dense = false;

@@ -104,6 +104,8 @@ struct LowerOptions {
 
 // Lower one parsed regex to IR (non-empty, unanchored match ends).
 void lower_regex(const Ast &ast, const LowerOptions &opt, RegexIR &ir);
+// Shift Rebalancing (Sec. 5.2): operand rewriting to a fixpoint + merging.
+void rebalance_regex(RegexIR &ir);
 // Compute margins, injection words and state slots.  Returns false if a
 // construct is not representable (message in why).
 bool analyze_regex(RegexIR &ir, std::string &why);

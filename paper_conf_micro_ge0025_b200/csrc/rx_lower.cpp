@@ -493,12 +493,14 @@ bool plan_groups(CompiledSet &cs, int group_size, int force_K, std::string &why)
       gr.slot_base.push_back(gr.nslots);
       gr.nslots += ir.nslots;
     }
-    int K = force_K;
-    if (K <= 0) {
-      K = 8;
-      for (int k : {1, 2, 4, 8})
-        if (4 * (L + R) <= 32 * k) { K = k; break; }
-    }
+    // K (words per lane): the smallest power of two >= the requested minimum
+    // (default 2: two independent words per lane per instruction, per-window
+    // costs amortised over 2048 positions) whose halo overhead is <= 25%
+    const int min_K = force_K > 0 ? force_K : 2;
+    int K = 8;
+    for (int k : {1, 2, 4, 8})
+      if (k >= min_K && 4 * (L + R) <= 32 * k) { K = k; break; }
+    if (K < min_K) K = min_K;
     if (L + R >= 32 * K) {
       why = "static span of a group exceeds the window (" + std::to_string(L + R) + " words)";
       return false;

@@ -240,7 +240,7 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
   rx::LowerOptions lo;
   lo.interval = o.interval == 0 ? 8 : (o.interval == UINT32_MAX ? 0 : (int)o.interval);
   if (o.flags & RX_F_NO_GUARDS) lo.interval = 0;
-  lo.rebalance = !(o.flags & RX_F_NO_REBALANCE);
+  lo.rebalance = (o.flags & RX_F_REBALANCE) && !(o.flags & RX_F_NO_REBALANCE);
   int max_regs = o.max_regs ? (int)o.max_regs : 128;
 
   auto *p = new rx_program();
@@ -269,6 +269,7 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
       return fail(RX_ETOOBIG, "pattern " + std::to_string(i) + ": expansion too large");
     }
     rx::lower_regex(*ast, lo, p->cs.irs[i]);
+    if (lo.rebalance) rx::rebalance_regex(p->cs.irs[i]);
     std::string why;
     if (!rx::analyze_regex(p->cs.irs[i], why)) {
       delete p;
@@ -421,7 +422,12 @@ rx_status launch(RxModule &m, CUfunction f, long long blocks, int warps_per_bloc
   Drv &d = drv();
   if (blocks <= 0) return RX_OK;
   if (blocks > 0x7fffffffLL) return fail(RX_EINVAL, "grid too large");
-  unsigned smem = (unsigned)(warps_per_block * (3 * m.nr_max * sizeof(unsigned long long) + 4 * m.ns_max * 4));
+  // must match the layout emitted in rx_codegen.cpp (accumulators | state |
+  // TMA window staging | mbarriers); the fix-up kernel uses the first two
+  const size_t wpb = (size_t)warps_per_block;
+  size_t bytes = wpb * 3 * m.nr_max * 8 + (((wpb * 4 * m.ns_max) + 3) & ~(size_t)3) * 4;
+  if (f == m.pass1) bytes += wpb * 4096 + wpb * 16;
+  unsigned smem = (unsigned)bytes;
   if (smem > 48 * 1024) d.FuncSetAttribute(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)smem);
   RxParamsHost local = prm;
   void *args[] = {&local};
