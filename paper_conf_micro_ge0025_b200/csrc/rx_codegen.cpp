@@ -338,20 +338,118 @@ struct RegexEmitter {
     }
   }
 
-  void emit_regex() {
-    os << "    // ---- regex member " << rloc << " (unguarded classes shared with the group)\n";
-    block(0, 3, "");
+  void emit_output(int in) {
     const Node &o = ir.nodes[ir.out];
-    if (o.op != Op::Zero) {
-      std::string R = nv(ir.out);
-      std::string m;
-      for (int i = 0; i < K; ++i) m += (i ? " | " : "") + ("(" + W(R, i) + " & c.cm[" + std::to_string(i) + "])");
-      os << "      if (c.want_dense || __any_sync(RX_FULL, (" << m << ") != 0u)) {\n";
-      os << "        V<" << K << "> ov;\n";
-      for (int i = 0; i < K; ++i) os << "        ov.w[" << i << "] = " << W(R, i) << ";\n";
-      os << "        rx_emit<" << K << ">(c, " << rloc << ", ov);\n";
-      os << "      }\n";
+    if (o.op == Op::Zero) return;
+    std::string I = ind(in);
+    std::string R = nv(ir.out);
+    std::string m;
+    for (int i = 0; i < K; ++i) m += (i ? " | " : "") + ("(" + W(R, i) + " & c.cm[" + std::to_string(i) + "])");
+    os << I << "if (c.want_dense || __any_sync(RX_FULL, (" << m << ") != 0u)) {\n";
+    os << I << "  V<" << K << "> ov;\n";
+    for (int i = 0; i < K; ++i) os << I << "  ov.w[" << i << "] = " << W(R, i) << ";\n";
+    os << I << "  rx_emit<" << K << ">(c, " << rloc << ", ov);\n";
+    os << I << "}\n";
+  }
+
+  // Two-phase emission: phase 1 holds every
+  // regex's unguarded head and the tests of its top-level zero-block guards,
+  // contiguous in the instruction stream; phase 2 holds the guarded bodies,
+  // the values depending on them and the output, and runs only for regexes
+  // whose guard fired (or that carry state through such values).
+  std::vector<char> post;   // top-level node depends on a guard result
+  bool has_guard = false, stateful_post = false;
+
+  void classify() {
+    post.assign(ir.nodes.size(), 0);
+    for (int id : ir.blocks[0].nodes) {
+      const Node &n = ir.nodes[id];
+      bool p = n.op == Op::Guard;
+      if (n.a >= 0 && post[n.a]) p = true;
+      if (n.b >= 0 && post[n.b]) p = true;
+      post[id] = p;
+      if (n.op == Op::Guard) has_guard = true;
+      if (p && (n.op == Op::MStar || n.op == Op::Loop)) stateful_post = true;
     }
+  }
+
+  std::string fire(int id) { return "f" + std::to_string(rloc) + "_" + std::to_string(id); }
+
+  // is top-level value `id` zero whenever no top-level guard fires (and no
+  // state flows in)?
+  bool zero_when_unfired(int id) {
+    const Node &n = ir.nodes[id];
+    switch (n.op) {
+      case Op::Guard: case Op::Zero: return true;
+      case Op::Ones: case Op::CC: case Op::Fr: return false;
+      case Op::And: return zero_when_unfired(n.a) || zero_when_unfired(n.b);
+      case Op::Or: case Op::Xor: return zero_when_unfired(n.a) && zero_when_unfired(n.b);
+      case Op::AndNot: case Op::Adv: case Op::Look: case Op::MStar: case Op::Loop: return zero_when_unfired(n.a);
+    }
+    return false;
+  }
+
+  // phase 1: returns the C expression "this regex needs phase 2"
+  std::string emit_phase1() {
+    classify();
+    os << "    // ---- regex member " << rloc << " (phase 1: unguarded head, guard tests)\n";
+    std::string need;
+    for (int id : ir.blocks[0].nodes) {
+      const Node &n = ir.nodes[id];
+      if (!post[id]) {
+        node(id, 2, "");
+        continue;
+      }
+      if (n.op == Op::Guard) {
+        std::vector<int> slots;
+        collect_slots(n.sub, slots);
+        std::string pend;
+        for (size_t i = 0; i < slots.size(); ++i) pend += (i ? " | " : "") + st(slots[i]);
+        if (post[n.a]) {
+          // a guard whose head depends on an earlier guard's result is tested
+          // inline in phase 2; phase 2 must run if state flows into it
+          if (!pend.empty()) need += (need.empty() ? "" : " || ") + ("((" + pend + ") != 0u)");
+          continue;
+        }
+        std::string cond = ir.nodes[n.a].op == Op::Ones ? "true" : any(nv(n.a));
+        decl(2, nv(id), [&](int) { return std::string("0u"); }, false);
+        os << "    const bool " << fire(id) << " = " << cond << (pend.empty() ? "" : " || ((" + pend + ") != 0u)")
+           << ";\n";
+        need += (need.empty() ? "" : " || ") + fire(id);
+      }
+    }
+    if (!has_guard) emit_output(2);
+    if (stateful_post) return "true";
+    // the output must be produced even when no guard fires if it has an
+    // unguarded contribution (e.g. an alternation with an unguarded branch)
+    if (has_guard && !zero_when_unfired(ir.out)) return "true";
+    return has_guard ? need : "";
+  }
+
+  // phase 2 (inside `if (need)`)
+  void emit_phase2() {
+    if (!has_guard) return;
+    os << "    // ---- regex member " << rloc << " (phase 2: guarded bodies)\n";
+    push();
+    for (int id : ir.blocks[0].nodes) {
+      if (!post[id]) continue;
+      const Node &n = ir.nodes[id];
+      if (n.op == Op::Guard && post[n.a]) {
+        node(id, 2, "");  // inline guard (head computed in phase 2)
+      } else if (n.op == Op::Guard) {
+        os << "    if (" << fire(id) << ") {\n";
+        push();
+        block(n.sub, 3, "");
+        pop();
+        std::string R = ir.nodes[n.res].op == Op::Zero ? "#0" : nv(n.res);
+        assign(3, nv(id), [&](int i) { return W(R, i); });
+        os << "    }\n";
+      } else {
+        node(id, 2, "");
+      }
+    }
+    emit_output(2);
+    pop();
   }
 };
 
@@ -400,9 +498,27 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
     for (int i = 0; i < g.K; ++i) os << "    const u32 vmw" << i << " = c.vm[" << i << "];\n";
     std::vector<std::map<TabKey, std::string>> ccs(1);
     std::vector<std::map<std::vector<uint64_t>, std::string>> sets(1);
+    std::vector<std::unique_ptr<RegexEmitter>> ems;
+    std::vector<std::string> needs;
     for (size_t m = 0; m < g.regexes.size(); ++m) {
-      RegexEmitter em(os, cs.irs[g.regexes[m]], g.K, (int)m, g.slot_base[m], ccs, sets);
-      em.emit_regex();
+      ems.emplace_back(new RegexEmitter(os, cs.irs[g.regexes[m]], g.K, (int)m, g.slot_base[m], ccs, sets));
+      needs.push_back(ems.back()->emit_phase1());
+    }
+    std::string any_need;
+    for (size_t m = 0; m < needs.size(); ++m)
+      if (!needs[m].empty()) {
+        os << "    const bool need" << m << " = " << needs[m] << ";\n";
+        any_need += (any_need.empty() ? "" : " || ") + std::string("need") + std::to_string(m);
+      }
+    if (!any_need.empty()) {
+      os << "    if (" << any_need << ") {\n";
+      for (size_t m = 0; m < needs.size(); ++m)
+        if (!needs[m].empty()) {
+          os << "    if (need" << m << ") {\n";
+          ems[m]->emit_phase2();
+          os << "    }\n";
+        }
+      os << "    }\n";
     }
     os << "  }\n};\n";
     os << "extern \"C\" __device__ __noinline__ void rx_seg_" << gi
