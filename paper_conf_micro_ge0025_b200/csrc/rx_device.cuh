@@ -177,6 +177,7 @@ struct RxParams {
   int aligned;              // in is 16-byte aligned
   int mode;                 // 0 = pass 1, 1 = fix-up with stored segment states, 2 = rematch
   int accumulate;           // counts/digests are added to (else the host zeroed them)
+  int lockstep;             // pass 1: one CTA barrier per window (warps of a group stay in step)
 };
 
 template <int K> DEV void rx_load_window(const RxParams &p, Ctx<K> &c, u32 (&pl)[8][K], i64 fword) {
@@ -405,6 +406,7 @@ DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned
     }
     __syncwarp();
     const RxRange ir = rx_interior(p);
+    const bool lockstep = p.lockstep != 0;
     bool issued0 = false, issued1 = false;
     u32 ph0 = 0, ph1 = 0;
     if (w_begin < w_end) {
@@ -455,7 +457,7 @@ DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned
         nst = t;
         __syncwarp();
       }
-      __syncthreads();
+      if (lockstep) __syncthreads();
     }
     if (!live) return;
     if (NS > 0) {
@@ -503,7 +505,7 @@ DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned
       nst = t;
       __syncwarp();
     }
-    __syncthreads();
+    if (p.lockstep) __syncthreads();
   }
   if (!live) return;
   if (NS > 0) {

@@ -375,6 +375,7 @@ struct RxParamsHost {  // must mirror RxParams in rx_device.cuh
   int aligned;
   int mode;
   int accumulate;
+  int lockstep;
 };
 
 rx_status ensure_loaded(rx_program *p, int &device) {
@@ -481,6 +482,10 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
   prm.st_assumed = (const unsigned int *)st_assumed;
   prm.aligned = (((uintptr_t)d_input) & 15) == 0 ? 1 : 0;
   prm.accumulate = accumulate;
+  {
+    const char *e = getenv("RX_LOCKSTEP");  // experiment knob: 0 = no per-window CTA barrier
+    prm.lockstep = (e && *e == '0') ? 0 : 1;
+  }
   static unsigned int dummy_status_host = 0;
   (void)dummy_status_host;
   unsigned int *status_scratch = nullptr;
