@@ -73,6 +73,8 @@ typedef struct {
                                 ILP only (no shift barriers at warp scope) -- see DESIGN.md */
 #define RX_F_NO_GUARDS 2u    /* disable Zero Block Skipping (Sec. 6) */
 #define RX_F_NO_CACHE 4u     /* do not read/write the on-disk cubin cache */
+#define RX_F_NO_PREFILTER 16u /* disable the cross-regex literal prefilter: every group
+                                 runs every window, gated only by Zero Block Skipping (Sec. 6) */
 
 /* Compile n patterns (byte strings, not NUL-terminated).  On error returns
  * the status and, if err != NULL, fills it.  *out owns everything. */

@@ -489,35 +489,45 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
        << ", NR = " << g.regexes.size() << ", SBASE = " << sbase << ", NG = " << G << ", GID = " << gi
        << ", NSMAX = " << nsmax << ";\n";
     os << "  static DEV const int *rid() { return rx_rid_" << gi << "; }\n";
+    os << "  static constexpr unsigned ALWAYS = " << g.always << "u;\n";
+    os << "  static constexpr bool PF = " << (cs.use_pf ? "true" : "false") << ";\n";
+    // rmask: members whose prefilter factor occurs in the window frame
+    // (rx_prefilter); members without a factor (ALWAYS) and members carrying
+    // state into the window run regardless
     os << "  static DEV void body(Ctx<" << g.K << "> &c, const u32 (&pl)[8][" << g.K
-       << "], const u32 *st, u32 *nst) {\n";
-    os << "    (void)st; (void)nst;\n";
+       << "], const u32 *st, u32 *nst, const u32 rmask) {\n";
+    os << "    (void)st; (void)nst; (void)rmask;\n";
     os << "    const u32 lane = c.lane; const int cw = (int)c.cw; (void)cw;\n";
     for (int k = 0; k < 8; ++k)
       for (int i = 0; i < g.K; ++i) os << "    const u32 b" << k << "w" << i << " = pl[" << k << "][" << i << "];\n";
     for (int i = 0; i < g.K; ++i) os << "    const u32 vmw" << i << " = c.vm[" << i << "];\n";
     std::vector<std::map<TabKey, std::string>> ccs(1);
     std::vector<std::map<std::vector<uint64_t>, std::string>> sets(1);
-    std::vector<std::unique_ptr<RegexEmitter>> ems;
-    std::vector<std::string> needs;
+    // one block per member: its unguarded head and guard tests (phase 1),
+    // then its guarded bodies (phase 2) if a guard fired
     for (size_t m = 0; m < g.regexes.size(); ++m) {
-      ems.emplace_back(new RegexEmitter(os, cs.irs[g.regexes[m]], g.K, (int)m, g.slot_base[m], ccs, sets));
-      needs.push_back(ems.back()->emit_phase1());
-    }
-    std::string any_need;
-    for (size_t m = 0; m < needs.size(); ++m)
-      if (!needs[m].empty()) {
-        os << "    const bool need" << m << " = " << needs[m] << ";\n";
-        any_need += (any_need.empty() ? "" : " || ") + std::string("need") + std::to_string(m);
-      }
-    if (!any_need.empty()) {
-      os << "    if (" << any_need << ") {\n";
-      for (size_t m = 0; m < needs.size(); ++m)
-        if (!needs[m].empty()) {
-          os << "    if (need" << m << ") {\n";
-          ems[m]->emit_phase2();
-          os << "    }\n";
+      const RegexIR &ir = cs.irs[g.regexes[m]];
+      RegexEmitter em(os, ir, g.K, (int)m, g.slot_base[m], ccs, sets);
+      std::string run;
+      if ((g.always >> m) & 1u) {
+        run = "true";
+      } else {
+        run = "((rmask >> " + std::to_string(m) + ") & 1u)";
+        if (ir.nslots > 0) {
+          std::string pend;
+          for (int sl = 0; sl < ir.nslots; ++sl) pend += (sl ? " | " : "") + em.st(sl);
+          run += " || ((" + pend + ") != 0u)";
         }
+      }
+      os << "    if (" << run << ") {\n";
+      em.push();
+      std::string need = em.emit_phase1();
+      if (!need.empty()) {
+        os << "    if (" << need << ") {\n";
+        em.emit_phase2();
+        os << "    }\n";
+      }
+      em.pop();
       os << "    }\n";
     }
     os << "  }\n};\n";
@@ -571,6 +581,9 @@ std::string emit_kernel_unit(CompiledSet &cs) {
         "  switch (g) {\n";
   for (int gi = 0; gi < G; ++gi) os << "    case " << gi << ": rx_seg_" << gi << "(p, (int)seg); break;\n";
   os << "    default: break;\n  }\n}\n";
+  if (cs.use_pf)
+    os << "\nextern \"C\" __global__ void __launch_bounds__(512, 1) rx_prefilter(const RxParams p) {\n"
+          "  rx_prefilter_run(p, RX_NG);\n}\n";
   os << "\nextern \"C\" __global__ void __launch_bounds__(128) rx_fixup(const RxParams p) {\n"
         "  const int warp = threadIdx.x >> 5;\n"
         "  const int wpb = blockDim.x >> 5;\n"

@@ -178,6 +178,17 @@ struct RxParams {
   int mode;                 // 0 = pass 1, 1 = fix-up with stored segment states, 2 = rematch
   int accumulate;           // counts/digests are added to (else the host zeroed them)
   int lockstep;             // pass 1: one CTA barrier per window (warps of a group stay in step)
+  // cross-regex prefilter (rx_prefilter below)
+  const u32 *pf_l1;         // [2048] bigram bitmap (last two bytes of every factor gram)
+  const u32 *pf_eoff;       // [65537] bigram -> entry range
+  const uint4 *pf_ent;      // {gram, mask, factor id, k}
+  const u32 *pf_fgoff;      // [nfactor+1] factor -> (group, member mask) range
+  const u32 *pf_fgent;      // {group, member mask}
+  u32 *pf_gbits;            // [NG][ntiles]: bit b of word t = factor of the group in block 32t+b
+  unsigned short *pf_blist; // [nblk][16]: hit count, then up to 15 factor ids (written for blocks with hits)
+  i64 pf_ntiles;
+  int pf_on;
+  int pf_aligned;           // in + avail_lo is 16-byte aligned
 };
 
 template <int K> DEV void rx_load_window(const RxParams &p, Ctx<K> &c, u32 (&pl)[8][K], i64 fword) {
@@ -384,10 +395,19 @@ DEV void rx_mbar_wait(u64 *bar, u32 phase) {
 // Runs one group (traits G) over one segment (pass 1).  Windows of groups
 // with K <= 2 are staged through shared memory by TMA bulk copies issued
 // one window ahead; wider groups prefetch into registers.
+template <class G> DEV void rx_run_segment_pf(const RxParams &p, int seg, u64 *acc, u32 *sst);
+
 template <class G>
 DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *tbuf, u64 *bars) {
   constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS;
   constexpr u32 WB = 1024u * K;  // window bytes
+  if constexpr (G::PF) {
+    (void)tbuf;
+    (void)bars;
+    (void)WB;
+    rx_run_segment_pf<G>(p, seg, acc, sst);
+    return;
+  }
   if constexpr (K <= 2) {
     const i64 len_words = rx_div_up(p.len, 32);
     const i64 nwin = rx_div_up(len_words, Bw);
@@ -451,7 +471,7 @@ DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned
         rx_unpack<K>(p, ir, c, xr, pl, fword);
         rx_commit_mask(p, ir, c, Lw, fword);
         if (NS > 0) rx_state_zero(nst, NS, c.lane);
-        G::body(c, pl, st, nst);
+        G::body(c, pl, st, nst, ~0u);
         u32 *t = st;
         st = nst;
         nst = t;
@@ -499,7 +519,7 @@ DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned
       if (w + 1 < w_end) rx_fetch<K>(p, ir, c.lane, xr, fword + Bw);  // prefetch the next window
       rx_commit_mask(p, ir, c, Lw, fword);
       if (NS > 0) rx_state_zero(nst, NS, c.lane);
-      G::body(c, pl, st, nst);
+      G::body(c, pl, st, nst, ~0u);
       u32 *t = st;
       st = nst;
       nst = t;
@@ -559,12 +579,12 @@ DEV void rx_fixup_group(const RxParams &p, u64 *acc, u32 *sst) {
       c.sign = ~0ull;
       c.want_dense = false;
       rx_state_zero(t1, NS, c.lane);
-      G::body(c, pl, old, t1);
+      G::body(c, pl, old, t1, ~0u);
       // new run: add, rewrite dense words
       c.sign = 1ull;
       c.want_dense = p.dense != nullptr;
       rx_state_zero(t2, NS, c.lane);
-      G::body(c, pl, tru, t2);
+      G::body(c, pl, tru, t2, ~0u);
       __syncwarp();
       rx_state_copy(old, t1, NS, c.lane);
       rx_state_copy(tru, t2, NS, c.lane);
@@ -579,6 +599,219 @@ DEV void rx_fixup_group(const RxParams &p, u64 *acc, u32 *sst) {
     }
     if (seg == nseg - 1 && p.st_out && (p.mode == 1 || !conv))
       for (int s = (int)c.lane; s < NS; s += 32) p.st_out[G::SBASE + s] = tru[s];
+  }
+  rx_flush<G>(p, c);
+}
+
+// ---------------------------------------------------------------------------
+// Cross-regex prefilter.
+// One streaming pass over the input: for every position q the 4 bytes ending
+// at q form x (little-endian, byte q on top); its last two bytes index a
+// 65,536-bit bigram bitmap held in shared memory; on a hit the (few) factor
+// grams ending in that bigram are verified exactly against x.  A tile of 32
+// blocks of 1 KiB is owned by one CTA, which records per block the factor
+// ids found (deduplicated, up to 15) and per group a 32-bit word with one bit
+// per block in which one of the group's factors occurs.
+// ---------------------------------------------------------------------------
+#define RX_PF_BLK 1024
+#define RX_PF_TILE 32768
+
+DEV void rx_pf_hit(const RxParams &p, u32 *gt, u32 *blc, unsigned short *blf, u32 x, i64 q, i64 tile_lo) {
+  const u32 bg = x >> 16;
+  const u32 e1 = __ldg(&p.pf_eoff[bg + 1]);
+  for (u32 e = __ldg(&p.pf_eoff[bg]); e < e1; ++e) {
+    const uint4 en = __ldg(&p.pf_ent[e]);
+    if ((x & en.y) != en.x || q - (i64)en.w + 1 < p.avail_lo) continue;
+    const int b = (int)((q - tile_lo) >> 10);
+    const u32 fid = en.z;
+    bool dup = false;
+    const u32 n0 = *(volatile u32 *)&blc[b];
+    for (u32 j = 0; j < n0 && j < 15u; ++j)
+      if (*(volatile unsigned short *)&blf[b * 15 + j] == (unsigned short)fid) dup = true;
+    if (dup) continue;
+    const u32 slot = atomicAdd(&blc[b], 1u);
+    if (slot < 15u) blf[b * 15 + slot] = (unsigned short)fid;
+    const u32 f1 = __ldg(&p.pf_fgoff[fid + 1]);
+    for (u32 j = __ldg(&p.pf_fgoff[fid]); j < f1; ++j) atomicOr(&gt[__ldg(&p.pf_fgent[2 * j])], 1u << b);
+  }
+}
+
+DEV u32 rx_load_u32_slow(const RxParams &p, i64 pos) {
+  u32 v = 0u;
+  for (int j = 0; j < 4; ++j) {
+    const i64 ps = pos + j;
+    if (ps >= p.avail_lo && ps < p.avail_hi) v |= (u32)p.in[ps] << (8 * j);
+  }
+  return v;
+}
+
+DEV void rx_prefilter_run(const RxParams &p, int NG) {
+  extern __shared__ __align__(16) u32 pf_smem[];
+  u32 *l1 = pf_smem;                 // 2048 words
+  u32 *blc = l1 + 2048;              // 32 hit counts
+  unsigned short *blf = reinterpret_cast<unsigned short *>(blc + 32);  // 32 x 15 factor ids
+  u32 *gt = blc + 32 + 240;          // NG words
+  const int tid = threadIdx.x, nt = blockDim.x;
+  for (int i = tid; i < 2048; i += nt) l1[i] = __ldg(&p.pf_l1[i]);
+  const u32 lane = rx_lane();
+  const i64 span = p.avail_hi - p.avail_lo;
+  const i64 ntiles = (span + RX_PF_TILE - 1) / RX_PF_TILE;
+  for (i64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    for (int i = tid; i < NG; i += nt) gt[i] = 0u;
+    if (tid < 32) blc[tid] = 0u;
+    __syncthreads();
+    const i64 tile_lo = p.avail_lo + t * RX_PF_TILE;
+    for (int j = 0; j < RX_PF_TILE / 16; j += nt) {
+      const i64 base = tile_lo + (i64)(j + tid) * 16;
+      u32 w[5];
+      if (p.pf_aligned && base + 16 <= p.avail_hi) {
+        const uint4 v = __ldg(reinterpret_cast<const uint4 *>(p.in + base));
+        w[1] = v.x; w[2] = v.y; w[3] = v.z; w[4] = v.w;
+      } else {
+#pragma unroll
+        for (int m = 0; m < 4; ++m) w[m + 1] = rx_load_u32_slow(p, base + 4 * m);
+      }
+      w[0] = __shfl_up_sync(RX_FULL, w[4], 1);
+      if (lane == 0) w[0] = rx_load_u32_slow(p, base - 4);
+#pragma unroll
+      for (int m = 0; m < 4; ++m) {
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+          const u32 x = r == 3 ? w[m + 1] : __funnelshift_r(w[m], w[m + 1], 8 * (r + 1));
+          const u32 bg = x >> 16;
+          if ((l1[bg >> 5] >> (bg & 31)) & 1u) {
+            const i64 q = base + 4 * m + r;
+            if (q < p.avail_hi) rx_pf_hit(p, gt, blc, blf, x, q, tile_lo);
+          }
+        }
+      }
+    }
+    __syncthreads();
+    for (int i = tid; i < NG; i += nt) p.pf_gbits[(i64)i * p.pf_ntiles + t] = gt[i];
+    for (int i = tid; i < 32 * 16; i += nt) {
+      const int b = i >> 4, e = i & 15;
+      const u32 n = blc[b];
+      if (n == 0u) continue;
+      const i64 gb = t * 32 + b;
+      p.pf_blist[gb * 16 + e] = e == 0 ? (unsigned short)(n > 0xffffu ? 0xffffu : n) : blf[b * 15 + e - 1];
+    }
+    __syncthreads();
+  }
+}
+
+// first block >= b0 (and <= bmax) whose bit is set in the group's bitmap;
+// returns bmax + 1 if none (warp-uniform)
+DEV i64 rx_pf_next(const u32 *gb, i64 b0, i64 bmax, u32 lane) {
+  for (i64 w0 = b0 >> 5; w0 <= (bmax >> 5); w0 += 32) {
+    const i64 wi = w0 + lane;
+    u32 v = wi <= (bmax >> 5) ? gb[wi] : 0u;
+    if (wi == (b0 >> 5)) v &= RX_FULL << (b0 & 31);
+    const u32 bal = __ballot_sync(RX_FULL, v != 0u);
+    if (bal) {
+      const int l = __ffs(bal) - 1;
+      const u32 vv = __shfl_sync(RX_FULL, v, l);
+      const i64 b = (w0 + l) * 32 + (__ffs(vv) - 1);
+      return b <= bmax ? b : bmax + 1;
+    }
+  }
+  return bmax + 1;
+}
+
+DEV i64 rx_floor_div(i64 a, i64 b) { return a >= 0 ? a / b : -((-a + b - 1) / b); }
+
+// Pass 1 with the prefilter: windows whose frame holds no factor of the group
+// and into which no state flows are skipped without loading a byte; the
+// others run only the members whose factor occurs in the frame, that carry
+// state, or that have no factor (G::ALWAYS).
+template <class G> DEV void rx_run_segment_pf(const RxParams &p, int seg, u64 *acc, u32 *sst) {
+  constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS;
+  const i64 len_words = rx_div_up(p.len, 32);
+  const i64 nwin = rx_div_up(len_words, Bw);
+  const i64 w_begin = (i64)seg * p.sw;
+  const bool live = w_begin < nwin || seg == 0;
+  const i64 w_end = !live ? w_begin : (w_begin + p.sw < nwin ? w_begin + p.sw : nwin);
+  Ctx<K> c;
+  rx_ctx_init<G>(p, c, acc);
+  u32 pl[8][K];
+  u32 xr[K][8];
+  u32 *st = sst, *nst = sst + G::NSMAX;
+  for (int s = (int)c.lane; s < NS; s += 32) st[s] = (seg == 0 && p.st_in) ? p.st_in[G::SBASE + s] : 0u;
+  __syncwarp();
+  const RxRange ir = rx_interior(p);
+  const u32 *gb = p.pf_gbits + (i64)G::GID * p.pf_ntiles;
+  auto frame_blocks = [&](i64 w, i64 &b0, i64 &b1) {
+    i64 flo = (w * Bw - Lw) * 32, fhi = flo + 1024 * K;
+    if (flo < p.avail_lo) flo = p.avail_lo;
+    if (fhi > p.avail_hi) fhi = p.avail_hi;
+    if (fhi <= flo) fhi = flo + 1;
+    b0 = (flo - p.avail_lo) >> 10;
+    b1 = (fhi - 1 - p.avail_lo) >> 10;
+  };
+  i64 bmax = 0;
+  if (w_begin < w_end) {
+    i64 t0;
+    frame_blocks(w_end - 1, t0, bmax);
+  }
+  i64 w = w_begin;
+  while (w < w_end) {
+    i64 b0, b1;
+    frame_blocks(w, b0, b1);
+    bool pend = false;
+    if (NS > 0) {
+      bool any = false;
+      for (int s = (int)c.lane; s < NS; s += 32) any = any || st[s] != 0u;
+      pend = __any_sync(RX_FULL, any);
+    }
+    if (!pend && G::ALWAYS == 0u) {
+      const i64 b = rx_pf_next(gb, b0, bmax, c.lane);
+      if (b > b1) {
+        if (b > bmax) break;
+        // the first window whose frame reaches block b
+        const i64 pos = p.avail_lo + b * RX_PF_BLK;
+        const i64 wn = rx_floor_div(rx_floor_div(pos, 32) + Lw - 32 * K, Bw) + 1;
+        w = wn > w + 1 ? wn : w + 1;
+        continue;
+      }
+    }
+    // members whose factor occurs in one of the frame's blocks
+    u32 mine = 0u;
+    for (i64 b = b0; b <= b1; ++b) {
+      if (!((gb[b >> 5] >> (b & 31)) & 1u)) continue;
+      const unsigned short *L = p.pf_blist + b * 16;
+      const u32 n = L[0];
+      if (n > 15u) {
+        mine = RX_FULL;
+        break;
+      }
+      if (c.lane < n) {
+        const u32 fid = L[1 + c.lane];
+        const u32 f1 = __ldg(&p.pf_fgoff[fid + 1]);
+        for (u32 j = __ldg(&p.pf_fgoff[fid]); j < f1; ++j)
+          if (__ldg(&p.pf_fgent[2 * j]) == (u32)G::GID) mine |= __ldg(&p.pf_fgent[2 * j + 1]);
+      }
+    }
+    const u32 rmask = __reduce_or_sync(RX_FULL, mine);
+    const i64 cstart = w * Bw;
+    const i64 fword = cstart - Lw;
+    c.cw = (u32)((len_words - cstart) < Bw ? (len_words - cstart) : Bw);
+    c.word0 = fword;
+    rx_fetch<K>(p, ir, c.lane, xr, fword);
+    rx_unpack<K>(p, ir, c, xr, pl, fword);
+    rx_commit_mask(p, ir, c, Lw, fword);
+    if (NS > 0) rx_state_zero(nst, NS, c.lane);
+    G::body(c, pl, st, nst, rmask);
+    u32 *t = st;
+    st = nst;
+    nst = t;
+    __syncwarp();
+    ++w;
+  }
+  if (!live) return;
+  if (NS > 0) {
+    u32 *dst = p.seg_state + ((i64)seg * G::NG + G::GID) * G::NSMAX;
+    for (int s = (int)c.lane; s < NS; s += 32) dst[s] = st[s];
+    if (p.st_out && w_end == nwin)
+      for (int s = (int)c.lane; s < NS; s += 32) p.st_out[G::SBASE + s] = st[s];
   }
   rx_flush<G>(p, c);
 }

@@ -116,6 +116,7 @@ std::string dump_ir(const RegexIR &ir);
 // ----------------------------------------------------------------------------
 struct Group {
   std::vector<int> regexes;  // global regex ids
+  uint32_t always = 0;       // members without a prefilter factor (run in every window)
   int K = 1;                 // words per lane per window
   int Lw = 0, Rw = 0, Bw = 0;  // window: left halo words, right halo words, committed words (32K = Lw+Bw+Rw)
   int nslots = 0;
@@ -123,7 +124,28 @@ struct Group {
   double cost = 0;
 };
 
+// Cross-regex literal prefilter (rx_prefilter.cpp).
+struct FactorGram {
+  uint32_t gram, mask;  // bytes of the k-gram in the top k bytes of a little-endian u32 window
+  int k;
+  bool operator==(const FactorGram &o) const { return gram == o.gram && mask == o.mask; }
+};
+struct Factor {
+  std::vector<FactorGram> grams;
+  double score = 0;  // estimated occurrences per position (ranking only)
+};
+struct Prefilter {
+  int nfactor = 0;
+  std::vector<uint32_t> l1, e_off, ent, fg_off, fg_ent;
+};
+// Returns false if the regex has no usable factor (it then always runs).
+bool regex_factor(const Ast &a, Factor &f);
+
 struct CompiledSet {
+  std::vector<int> factor_of;     // per regex: factor id or -1 (always runs)
+  std::vector<Factor> factors;
+  Prefilter pf;
+  bool use_pf = false;
   std::vector<RegexIR> irs;
   std::vector<Group> groups;
   std::string source;  // generated CUDA C
@@ -135,5 +157,6 @@ struct CompiledSet {
 std::string emit_group_unit(CompiledSet &cs, int gi);
 std::string emit_kernel_unit(CompiledSet &cs);
 bool plan_groups(CompiledSet &cs, int group_size, int force_K, std::string &why);
+void build_prefilter(CompiledSet &cs);
 
 }  // namespace rx

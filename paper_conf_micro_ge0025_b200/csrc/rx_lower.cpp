@@ -460,19 +460,34 @@ bool plan_groups(CompiledSet &cs, int group_size, int force_K, std::string &why)
   std::vector<int> order(n);
   for (int i = 0; i < n; ++i) order[i] = i;
   auto span = [&](int r) { return (cs.irs[r].lb + 31) / 32 + (std::max(cs.irs[r].rb, cs.irs[r].rb_state) + 31) / 32; };
-  std::stable_sort(order.begin(), order.end(), [&](int a, int b) { return span(a) < span(b); });
+  // window-width class first (a group's geometry must fit every member),
+  // then -- with the prefilter -- members without a factor apart from the
+  // others (their groups run every window), and members sharing a factor
+  // together (one factor hit then wakes one group)
+  auto kclass = [&](int r) {
+    const int w = span(r);
+    for (int k : {2, 4, 8})
+      if (4 * w <= 32 * k) return k;
+    return 16;
+  };
+  auto fac = [&](int r) { return cs.factor_of.empty() ? -1 : cs.factor_of[r]; };
+  std::stable_sort(order.begin(), order.end(), [&](int a, int b) {
+    if (kclass(a) != kclass(b)) return kclass(a) < kclass(b);
+    if ((fac(a) < 0) != (fac(b) < 0)) return fac(a) < 0;
+    if (fac(a) != fac(b)) return fac(a) < fac(b);
+    return span(a) < span(b);
+  });
   size_t total_instr = 0;
   for (auto &r : cs.irs) total_instr += r.n_instr;
-  if (group_size <= 0) {
-    // aim for <= ~64 regexes and a bounded code size per group
-    group_size = 32;
-  }
+  if (group_size <= 0 || group_size > 32) group_size = 32;  // member masks are 32-bit
   const size_t max_instr = 1500;  // bounds one NVRTC unit (compile time) and the group's code size
   cs.groups.clear();
   Group g;
   size_t gi = 0;
   for (int r : order) {
-    if (!g.regexes.empty() && ((int)g.regexes.size() >= group_size || gi + cs.irs[r].n_instr > max_instr)) {
+    const bool split_always = !g.regexes.empty() && (fac(g.regexes.back()) < 0) != (fac(r) < 0);
+    if (!g.regexes.empty() &&
+        ((int)g.regexes.size() >= group_size || gi + cs.irs[r].n_instr > max_instr || split_always)) {
       cs.groups.push_back(g);
       g = Group();
       gi = 0;
@@ -486,8 +501,10 @@ bool plan_groups(CompiledSet &cs, int group_size, int force_K, std::string &why)
     int L = 0, R = 0;
     gr.nslots = 0;
     gr.slot_base.clear();
+    gr.always = 0;
     for (int r : gr.regexes) {
       const RegexIR &ir = cs.irs[r];
+      if (fac(r) < 0) gr.always |= 1u << gr.slot_base.size();
       L = std::max(L, (ir.lb + 31) / 32);
       R = std::max(R, (std::max(ir.rb, ir.rb_state) + 31) / 32);
       gr.slot_base.push_back(gr.nslots);

@@ -14,6 +14,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <fstream>
+#include <map>
 #include <mutex>
 #include <sstream>
 #include <string>
@@ -184,7 +185,10 @@ struct RxModule {
   // loaded (device-specific)
   int device = -1;
   CUmodule mod = nullptr;
-  CUfunction pass1 = nullptr, fixup = nullptr;
+  CUfunction pass1 = nullptr, fixup = nullptr, prefilter = nullptr;
+  // prefilter tables on the device (uploaded at load)
+  void *pf_mem = nullptr;
+  const void *pf_l1 = nullptr, *pf_eoff = nullptr, *pf_ent = nullptr, *pf_fgoff = nullptr, *pf_fgent = nullptr;
 };
 
 struct rx_program {
@@ -211,7 +215,7 @@ const char *rx_program_source(const rx_program *p) { return p ? p->all_source.c_
 uint32_t rx_kernels_per_match(const rx_program *p) {
   uint32_t n = 0;
   if (p)
-    for (auto &m : p->mods) n += 1 + (m.any_state ? 1 : 0);
+    for (auto &m : p->mods) n += 1 + (m.any_state ? 1 : 0) + (p->cs.use_pf ? 1 : 0);
   return n;
 }
 const char *rx_program_info(const rx_program *p) { return p ? p->info.c_str() : ""; }
@@ -225,6 +229,7 @@ void rx_free(rx_program *p) {
       cudaGetDevice(&cur);
       if (cur != m.device) cudaSetDevice(m.device);
       d.ModuleUnload(m.mod);
+      if (m.pf_mem) cudaFree(m.pf_mem);
       if (cur != m.device && cur >= 0) cudaSetDevice(cur);
     }
   delete p;
@@ -246,6 +251,9 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
   auto *p = new rx_program();
   p->n_regex = n_patterns;
   p->cs.irs.resize(n_patterns);
+  p->cs.factor_of.assign(n_patterns, -1);
+  const bool use_pf = !(o.flags & RX_F_NO_PREFILTER);
+  std::map<std::vector<uint32_t>, int> factor_ix;
   for (uint32_t i = 0; i < n_patterns; ++i) {
     std::string pat(patterns[i], pattern_lens[i]);
     rx::ParseError pe;
@@ -268,6 +276,23 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
       delete p;
       return fail(RX_ETOOBIG, "pattern " + std::to_string(i) + ": expansion too large");
     }
+    {
+      rx::Factor f;
+      int fid = -1;
+      if (use_pf && rx::regex_factor(*ast, f)) {
+        std::vector<uint32_t> key;
+        for (auto &g : f.grams) key.insert(key.end(), {g.gram, g.mask});
+        auto it = factor_ix.find(key);
+        if (it == factor_ix.end()) {
+          fid = (int)p->cs.factors.size();
+          factor_ix[key] = fid;
+          p->cs.factors.push_back(f);
+        } else {
+          fid = it->second;
+        }
+      }
+      p->cs.factor_of[i] = fid;
+    }
     rx::lower_regex(*ast, lo, p->cs.irs[i]);
     if (lo.rebalance) rx::rebalance_regex(p->cs.irs[i]);
     std::string why;
@@ -286,6 +311,8 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
     delete p;
     return fail(RX_ETOOBIG, why);
   }
+  p->cs.use_pf = !p->cs.factors.empty();
+  if (p->cs.use_pf) rx::build_prefilter(p->cs);
   // one relocatable NVRTC unit per group + the kernel unit, compiled in
   // parallel and linked into one module by nvJitLink
   int G = (int)p->cs.groups.size();
@@ -307,7 +334,22 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
     sbase += (uint32_t)g.nslots;
   }
   p->state_words = sbase;
-  for (uint32_t i = 0; i < n_patterns; ++i) info << "regex " << i << ":\n" << rx::dump_ir(p->cs.irs[i]);
+  info << "prefilter: " << (p->cs.use_pf ? "on" : "off") << ", factors=" << p->cs.factors.size() << "\n";
+  for (uint32_t i = 0; i < n_patterns; ++i) {
+    const int f = p->cs.factor_of[i];
+    info << "regex " << i << ": factor ";
+    if (f < 0) info << "none (always runs)";
+    else {
+      info << f << " (" << p->cs.factors[f].grams.size() << " grams, k=" << p->cs.factors[f].grams[0].k
+           << ", score=" << p->cs.factors[f].score << ") grams=";
+      char hx[24];
+      for (auto &g : p->cs.factors[f].grams) {
+        snprintf(hx, sizeof hx, "%08x/%d,", g.gram, g.k);
+        info << hx;
+      }
+    }
+    info << "\n" << rx::dump_ir(p->cs.irs[i]);
+  }
   p->info = info.str();
   std::vector<std::string> srcs(G + 1), cubins(G + 1), logs(G + 1);
   for (int gi = 0; gi < G; ++gi) srcs[gi] = rx::emit_group_unit(p->cs, gi);
@@ -376,6 +418,12 @@ struct RxParamsHost {  // must mirror RxParams in rx_device.cuh
   int mode;
   int accumulate;
   int lockstep;
+  const void *pf_l1, *pf_eoff, *pf_ent, *pf_fgoff, *pf_fgent;
+  unsigned int *pf_gbits;
+  unsigned short *pf_blist;
+  long long pf_ntiles;
+  int pf_on;
+  int pf_aligned;
 };
 
 rx_status ensure_loaded(rx_program *p, int &device) {
@@ -410,6 +458,28 @@ rx_status ensure_loaded(rx_program *p, int &device) {
     if (d.ModuleGetFunction(&m.pass1, m.mod, "rx_pass1") != CUDA_SUCCESS ||
         d.ModuleGetFunction(&m.fixup, m.mod, "rx_fixup") != CUDA_SUCCESS)
       return fail(RX_ECUDA, "kernel symbols missing");
+    if (p->cs.use_pf) {
+      if (d.ModuleGetFunction(&m.prefilter, m.mod, "rx_prefilter") != CUDA_SUCCESS)
+        return fail(RX_ECUDA, "rx_prefilter symbol missing");
+      const rx::Prefilter &pf = p->cs.pf;
+      const std::vector<uint32_t> *parts[] = {&pf.l1, &pf.e_off, &pf.ent, &pf.fg_off, &pf.fg_ent};
+      size_t off[5], total = 0;
+      for (int i = 0; i < 5; ++i) {
+        off[i] = total;
+        total += (4 * parts[i]->size() + 255) & ~(size_t)255;
+      }
+      if (cudaMalloc(&m.pf_mem, total + 256) != cudaSuccess) return fail(RX_ENOMEM, "prefilter tables");
+      for (int i = 0; i < 5; ++i)
+        if (!parts[i]->empty() &&
+            cudaMemcpy((char *)m.pf_mem + off[i], parts[i]->data(), 4 * parts[i]->size(), cudaMemcpyHostToDevice) !=
+                cudaSuccess)
+          return fail(RX_ECUDA, "prefilter table upload");
+      m.pf_l1 = (char *)m.pf_mem + off[0];
+      m.pf_eoff = (char *)m.pf_mem + off[1];
+      m.pf_ent = (char *)m.pf_mem + off[2];
+      m.pf_fgoff = (char *)m.pf_mem + off[3];
+      m.pf_fgent = (char *)m.pf_mem + off[4];
+    }
     m.device = device;
   }
   return RX_OK;
@@ -428,6 +498,7 @@ rx_status launch(RxModule &m, CUfunction f, long long blocks, int warps_per_bloc
   const size_t wpb = (size_t)warps_per_block;
   size_t bytes = wpb * 3 * m.nr_max * 8 + (((wpb * 4 * m.ns_max) + 3) & ~(size_t)3) * 4;
   if (f == m.pass1) bytes += wpb * 4096 + wpb * 16;
+  if (f == m.prefilter) bytes = 4 * (2048 + 32 + 240 + (size_t)(m.g_end - m.g_begin));
   unsigned smem = (unsigned)bytes;
   if (smem > 48 * 1024) d.FuncSetAttribute(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)smem);
   RxParamsHost local = prm;
@@ -530,7 +601,31 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
     }
     prm.seg_state = seg_state;
     prm.mode = 0;
+    void *pf_scratch = nullptr;
+    if (p->cs.use_pf) {
+      const long long span = prm.avail_hi - prm.avail_lo;
+      const long long ntiles = std::max<long long>(1, div_up(span, 32768));
+      const size_t gb_bytes = (size_t)4 * (size_t)ntiles * (size_t)mg;
+      const size_t bl_bytes = (size_t)ntiles * 32 * 32;
+      if (cudaMallocAsync(&pf_scratch, gb_bytes + bl_bytes + 256, stream) != cudaSuccess)
+        return fail(RX_ENOMEM, "prefilter scratch");
+      prm.pf_l1 = m.pf_l1;
+      prm.pf_eoff = m.pf_eoff;
+      prm.pf_ent = m.pf_ent;
+      prm.pf_fgoff = m.pf_fgoff;
+      prm.pf_fgent = m.pf_fgent;
+      prm.pf_gbits = (unsigned int *)pf_scratch;
+      prm.pf_blist = (unsigned short *)((char *)pf_scratch + ((gb_bytes + 255) & ~(size_t)255));
+      prm.pf_ntiles = ntiles;
+      prm.pf_on = 1;
+      prm.pf_aligned = (((uintptr_t)(d_input - halo_left)) & 15) == 0 ? 1 : 0;
+      prm.lockstep = 0;
+      s = launch(m, m.prefilter, std::min<long long>(ntiles, 148LL * 4), 16, prm, stream);
+      if (s != RX_OK) return s;
+    }
     s = launch(m, m.pass1, cpg * mg, kPass1Warps, prm, stream);
+    if (pf_scratch) cudaFreeAsync(pf_scratch, stream);
+    prm.pf_on = 0;
     if (s != RX_OK) return s;
     if (m.any_state) {
       prm.mode = 1;
