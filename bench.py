@@ -97,21 +97,34 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(self.rows)}
 
 
-def load_workload(config: str, rank: int = 0, world: int = 1):
+WORKLOADS = {
+    # name: (pattern builder, input builder(length, rank), default bytes per GPU, description)
+    "snort": (lambda: __import__("gen").snort_patterns(1000, 2)[0],
+              lambda n, r: __import__("gen").snort_input(n, seed=2 + 1000 * r), 256 << 20,
+              "snort-like 1k regexes x 256 MiB payloads"),
+    "clamav": (lambda: __import__("gen").clamav_brill_patterns(1000, 3)[0],
+               lambda n, r: __import__("gen").text_input(n, seed=3 + 1000 * r), 1 << 30,
+               "clamav/brill-like 2k regexes x 1 GiB text"),
+    "dotstar": (lambda: __import__("gen").dotstar_protomata_patterns(1000, 4)[0],
+                lambda n, r: __import__("gen").dotstar_input(n, seed=4 + 1000 * r), 1 << 30,
+                "dotstar/protomata-like 2k regexes x 1 GiB amino/long-line text"),
+    "multi": (lambda: __import__("gen").multi_patterns(2500),
+              lambda n, r: __import__("gen").multi_input(n, seed=5 + 1000 * r), 8 << 30,
+              "10k regexes (2.5k per family) x 8 GiB"),
+}
+
+
+def load_workload(config: str, length=None, rank: int = 0):
+    """(patterns, input u8 array, bytes, description) of a named workload."""
     import gen
     if config == "tiny":
-        return gen.tiny_patterns(), np.frombuffer(gen.tiny_input(), dtype=np.uint8), "tiny"
-    if config == "snort":
-        pats = gen.snort_patterns(1000, 2)[0]
-        length = 256 << 20
-        return pats, None, "snort-like 1k regexes x 256 MiB payloads"
-    raise SystemExit(f"unknown config {config}")
-
-
-def snort_chunk(rank: int, length: int):
-    import gen
-    # rank r's chunk of the stream: seed 2 for rank 0 (the N=1 workload)
-    return gen.snort_input(length, seed=2 + 1000 * rank)
+        data = np.frombuffer(gen.tiny_input(), dtype=np.uint8)
+        return gen.tiny_patterns(), data, data.size, "tiny"
+    if config not in WORKLOADS:
+        raise SystemExit(f"unknown config {config}")
+    pb, ib, n, desc = WORKLOADS[config]
+    n = int(length or n)
+    return pb(), ib(n, rank), n, desc
 
 
 # ---------------------------------------------------------------------------
@@ -137,9 +150,12 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    pats, data, name = load_workload(args.config)
-    if data is None:
-        data = snort_chunk(0, 16 << 20)
+    if args.config == "tiny":
+        pats, data, n, name = load_workload("tiny")
+    else:
+        pb, ib, n, name = WORKLOADS[args.config]
+        pats = pb()
+        data = ib(16 << 20, 0)
     rates = []
     samples = []
     for _ in range(args.warmup):
@@ -152,7 +168,7 @@ def run_reference(args):
     n, dt = samples[-1]
     line = {"metric": "input GB/s scanned per regex set", "value": gbs, "unit": "GB/s", "impl": "reference",
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": 1e3 * (256 << 20) / (gbs * 1e9), "higher_is_better": True, "scaling": "weak",
+            "ms_per_step": 1e3 * n / (gbs * 1e9), "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "u8", "data": "synthetic",
             "config": {"workload": name, "n_regex": len(pats), "input_bytes": 256 << 20},
             "cpu_baseline": {"value": gbs, "unit": "GB/s", "cores": thr, "kind": "oracle",
@@ -173,7 +189,8 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="snort")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--length-mib", type=int, default=256)
+    ap.add_argument("--length-mib", type=int, default=0, help="input bytes per GPU (default: the config's)")
+    ap.add_argument("--no-prefilter", action="store_true", help="ablation: RX_F_NO_PREFILTER")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -190,12 +207,10 @@ def main():
     dev = torch.device("cuda", local)
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
-    pats, data, name = load_workload(args.config)
-    if data is None:
-        data = snort_chunk(rank, args.length_mib << 20)
+    pats, data, nbytes, name = load_workload(args.config, (args.length_mib << 20) if args.length_mib else None, rank)
     nbytes = int(data.size)
     t0 = time.perf_counter()
-    prog = rx.Program(pats)
+    prog = rx.Program(pats, flags=rx.RX_F_NO_PREFILTER if args.no_prefilter else 0)
     compile_s = time.perf_counter() - t0
 
     host = torch.from_numpy(np.ascontiguousarray(data)).pin_memory()
@@ -222,10 +237,30 @@ def main():
         step_device()
     torch.cuda.synchronize(dev)
 
+    # inputs smaller than L2 (126 MB): flush L2 before every timed step and
+    # time the steps one by one (the flush stays outside the events)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev) if nbytes <= (128 << 20) else None
+
     def timed(fn, k):
         if world > 1:
             dist.barrier()
         torch.cuda.synchronize(dev)
+        if flush is not None:
+            tot = 0.0
+            for _ in range(k):
+                flush.fill_(1)
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(stream)
+                fn()
+                e1.record(stream)
+                torch.cuda.synchronize(dev)
+                tot += e0.elapsed_time(e1)
+            ms = tot / k
+            if world > 1:
+                t = torch.tensor([ms], device=dev)
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                ms = float(t.item())
+            return ms
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
         for _ in range(k):
@@ -258,7 +293,9 @@ def main():
         "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
         "config": {"workload": name, "n_regex": len(pats), "input_bytes_per_gpu": nbytes,
                    "groups": prog.n_groups, "outputs": "per-regex counts (dense streams off: 31 GiB at this size)",
-                   "l2": "input 256 MiB > 126 MB L2: no flush needed", "compile_s": round(compile_s, 1)},
+                   "l2": f"input {nbytes >> 20} MiB per GPU" + (" > 126 MB L2: no flush needed" if nbytes > (126 << 20)
+                                                                  else " < L2: L2 flushed between steps"),
+                   "prefilter": not args.no_prefilter, "compile_s": round(compile_s, 1)},
         "roofline": {"bound": "hbm", "achieved": gbs / world, "peak": hbm, "unit": "GB/s",
                      "frac": gbs / world / hbm, "traffic": None, "peak_source": hbm_src,
                      "note": "achieved = input bytes (read once) / step time of the fused pass; the kernel is "

@@ -396,3 +396,319 @@ CONFIGS["snort"] = {
     "len": 256 << 20,
     "desc": "Snort-like: 1,000 regexes over 256 MiB synthetic packet payloads (seed 2)",
 }
+
+
+# ---------------------------------------------------------------------------
+# config 3: ClamAV-like hex signatures + Brill-like word rules over text
+# (Table 1: ClamAV length mean 359.7 / SD 310.7 chars; Brill 44.4 /
+# 16.9)
+# ---------------------------------------------------------------------------
+def _syn_words(rng, n: int):
+    """n synthetic lowercase words (2-10 letters), deterministic."""
+    letters = b"etaoinshrdlcumwfgypbvkjxqz"
+    freq = np.array([12.7, 9.1, 8.2, 7.5, 7.0, 6.7, 6.3, 6.1, 6.0, 4.3, 4.0, 2.8, 2.8, 2.4, 2.4, 2.2, 2.0, 2.0, 1.9,
+                     1.5, 1.0, 0.8, 0.2, 0.2, 0.1, 0.1])
+    freq = freq / freq.sum()
+    out = set()
+    while len(out) < n:
+        k = int(rng.integers(2, 11))
+        out.add(bytes(letters[int(i)] for i in rng.choice(26, size=k, p=freq)))
+    return sorted(out)
+
+
+def _zipf_text(rng, length: int, words, s: float = 1.1, line: int = 80) -> np.ndarray:
+    ranks = np.arange(1, len(words) + 1, dtype=np.float64)
+    p = ranks ** (-s)
+    p /= p.sum()
+    punct = [b" ", b" ", b" ", b" ", b" ", b", ", b". ", b"; "]
+    out = bytearray()
+    col = 0
+    while len(out) < length:
+        idx = rng.choice(len(words), size=4096, p=p)
+        pk = rng.integers(0, len(punct), size=4096)
+        for i, j in zip(idx, pk):
+            w = words[int(i)] + punct[int(j)]
+            out += w
+            col += len(w)
+            if col >= line:
+                out += b"\n"
+                col = 0
+        if len(out) >= length:
+            break
+    return np.frombuffer(bytes(out[:length]), dtype=np.uint8).copy()
+
+
+_TEXT_WORDS_SEED = 33
+
+
+def text_words(n: int = 50000):
+    """n synthetic words in Zipf-rank order (a seeded permutation)."""
+    rng = np.random.default_rng(_TEXT_WORDS_SEED)
+    w = _syn_words(rng, n)
+    return [w[int(i)] for i in rng.permutation(len(w))]
+
+
+def clamav_patterns(n: int = 1000, seed: int = 3):
+    """Hex byte signatures, length lognormal mean 360 / SD 311 chars clipped to
+    [16, 2048]; 10% with '.' or '.{0,32}' gaps."""
+    rng = np.random.default_rng(seed)
+    pats, samplers = [], []
+    for _ in range(n):
+        chars = _lognormal_len(rng, 360, 311, lo=16, hi=2048)
+        nbytes = max(4, chars // 4)
+        toks = []
+        gap = rng.random() < 0.10
+        left = nbytes
+        while left > 0:
+            seg = int(min(left, rng.integers(8, 40) if gap else left))
+            b = bytes(rng.integers(0, 256, size=seg, dtype=np.uint8))
+            toks.append(_Tok(b"".join(b"\\x%02x" % c for c in b), lambda g, b=b: b))
+            left -= seg
+            if gap and left > 0:
+                if rng.random() < 0.5:
+                    toks.append(_Tok(b".", lambda g: bytes([int(g.integers(0, 10))])))
+                else:
+                    k = int(rng.integers(1, 33))
+                    toks.append(_quantified(b".", lambda g: b"a", 0, k, b"{0,%d}" % k))
+        pats.append(b"".join(t.text for t in toks))
+        samplers.append(lambda g, toks=toks: b"".join(t.sample(g) for t in toks))
+    return pats, samplers
+
+
+def brill_patterns(n: int = 1000, seed: int = 3):
+    """Word-sequence rules (mean ~44 chars): alternations of words joined by
+    '[ ]+' and optional '[a-z]+' wildcards."""
+    rng = np.random.default_rng(seed * 101 + 7)
+    words = text_words()
+    top = words[:3000]
+    pats, samplers = [], []
+    for _ in range(n):
+        target = _lognormal_len(rng, 44.4, 16.9, lo=10, hi=160)
+        toks = []
+        size = 0
+        while size < target:
+            if toks:
+                toks.append(_Tok(b"[ ]+", lambda g: b" "))
+            r = rng.random()
+            if r < 0.5:
+                w = top[int(rng.integers(0, len(top)))]
+                t = _lit(w)
+            elif r < 0.8:
+                alts = [top[int(i)] for i in rng.integers(0, len(top), size=int(rng.integers(2, 5)))]
+                t = _alt_tok(alts)
+            else:
+                t = _Tok(b"[a-z]+", lambda g: bytes(b"abcdefghijklmnopqrstuvwxyz"[int(i)]
+                                                       for i in g.integers(0, 26, size=int(g.integers(1, 8)))))
+            toks.append(t)
+            size = sum(len(x.text) for x in toks)
+        pats.append(b"".join(t.text for t in toks))
+        samplers.append(lambda g, toks=toks: b"".join(t.sample(g) for t in toks))
+    return pats, samplers
+
+
+def clamav_brill_patterns(n_each: int = 1000, seed: int = 3):
+    a, sa = clamav_patterns(n_each, seed)
+    b, sb = brill_patterns(n_each, seed)
+    return a + b, sa + sb
+
+
+def text_input(length: int = 1 << 30, seed: int = 3, patterns_seed: int = 3, n_each: int = 1000,
+               plant_every: int = 1 << 20):
+    """Zipf(1.1) text over 50k synthetic words with punctuation and a newline
+    every ~80 chars; members of the pattern set planted about once per MiB."""
+    rng = np.random.default_rng(seed * 7919 + 3)
+    pool = _zipf_text(rng, min(length, 8 << 20) + 1, text_words())
+    reps = -(-length // pool.size)
+    if reps > 1:
+        offs = rng.integers(0, pool.size, size=reps)
+        buf = np.concatenate([np.roll(pool, -int(o)) for o in offs])[:length].copy()
+    else:
+        buf = pool[:length].copy()
+    _, samplers = clamav_brill_patterns(n_each, patterns_seed)
+    _plant(rng, buf, samplers, plant_every)
+    return buf
+
+
+CONFIGS["clamav"] = {
+    "patterns": lambda n=1000, seed=3: clamav_brill_patterns(n, seed)[0],
+    "input": lambda length=1 << 30, seed=3: text_input(length, seed),
+    "pattern_kw": ("n",),
+    "input_kw": ("length",),
+    "len": 1 << 30,
+    "desc": "ClamAV/Brill-like: 1,000 hex signatures + 1,000 word rules over 1 GiB text (seed 3)",
+}
+
+
+# ---------------------------------------------------------------------------
+# config 4: Dotstar-like + PROSITE/Protomata-like motifs (Table 1 Protomata
+# length mean 96.5 / SD 36.2, P:L393) over amino-acid text and long lines
+# ---------------------------------------------------------------------------
+_AMINO = b"ACDEFGHIKLMNPQRSTVWY"
+_AMINO_FREQ = np.array([8.25, 1.37, 5.45, 6.75, 3.86, 7.07, 2.27, 5.96, 5.84, 9.66, 2.42, 4.06, 4.70, 3.93, 5.53,
+                        6.56, 5.34, 6.87, 1.08, 2.92])
+_AMINO_FREQ = _AMINO_FREQ / _AMINO_FREQ.sum()
+_AMINO_CLASSES = [b"[ILMV]", b"[FYW]", b"[KR]", b"[DE]", b"[ST]", b"[AG]", b"[NQ]", b"[^P]", b"[^C]"]
+
+
+def _amino_class_members(text: bytes) -> bytes:
+    if text.startswith(b"[^"):
+        return bytes(c for c in _AMINO if c != text[2])
+    return text[1:-1]
+
+
+def dotstar_patterns(n: int = 1000, seed: int = 4):
+    """3-6 literal segments of 4-12 bytes joined by '.*' (p = 0.3), else by
+    '[^\\n]*' or '.{0,k}'."""
+    rng = np.random.default_rng(seed)
+    pats, samplers = [], []
+    alpha = b"abcdefghijklmnopqrstuvwxyzABCDEFGHIJKLMNOPQRSTUVWXYZ0123456789"
+    for _ in range(n):
+        toks = []
+        for si in range(int(rng.integers(3, 7))):
+            if si:
+                r = rng.random()
+                if r < 0.3:
+                    toks.append(_quantified(b".", lambda g: b"x", 0, -1, b"*"))
+                elif r < 0.65:
+                    toks.append(_quantified(rb"[^\n]", lambda g: b"y", 0, -1, b"*"))
+                else:
+                    k = int(rng.integers(1, 64))
+                    toks.append(_quantified(b".", lambda g: b"z", 0, k, b"{0,%d}" % k))
+            w = bytes(alpha[int(i)] for i in rng.integers(0, len(alpha), size=int(rng.integers(4, 13))))
+            toks.append(_lit(w))
+        pats.append(b"".join(t.text for t in toks))
+        samplers.append(lambda g, toks=toks: b"".join(t.sample(g) for t in toks))
+    return pats, samplers
+
+
+def protomata_patterns(n: int = 1000, seed: int = 4):
+    """PROSITE-like motifs over the 20 amino acids: letters, classes such as
+    [ILMV] and [^P], '.', '.{2,4}'; length mean 96.5 / SD 36.2 chars."""
+    rng = np.random.default_rng(seed * 101 + 9)
+    pats, samplers = [], []
+    for _ in range(n):
+        target = _lognormal_len(rng, 96.5, 36.2, lo=12, hi=300)
+        toks = []
+        size = 0
+        while size < target:
+            r = rng.random()
+            if r < 0.45:
+                c = bytes([_AMINO[int(rng.choice(20, p=_AMINO_FREQ))]])
+                t = _lit(c)
+            elif r < 0.8:
+                cl = _AMINO_CLASSES[int(rng.integers(0, len(_AMINO_CLASSES)))]
+                m = _amino_class_members(cl)
+                t = _Tok(cl, lambda g, m=m: bytes([m[int(g.integers(0, len(m)))]]))
+            elif r < 0.9:
+                t = _Tok(b".", lambda g: bytes([_AMINO[int(g.integers(0, 20))]]))
+            else:
+                lo = int(rng.integers(1, 4))
+                hi = lo + int(rng.integers(1, 4))
+                t = _quantified(b".", lambda g: bytes([_AMINO[int(g.integers(0, 20))]]), lo, hi,
+                                b"{%d,%d}" % (lo, hi))
+            toks.append(t)
+            size += len(t.text)
+        pats.append(b"".join(t.text for t in toks))
+        samplers.append(lambda g, toks=toks: b"".join(t.sample(g) for t in toks))
+    return pats, samplers
+
+
+def dotstar_protomata_patterns(n_each: int = 1000, seed: int = 4):
+    a, sa = dotstar_patterns(n_each, seed)
+    b, sb = protomata_patterns(n_each, seed)
+    return a + b, sa + sb
+
+
+def amino_lines(rng, length: int) -> np.ndarray:
+    """Amino-acid text in lines of 60-80 letters (background frequencies)."""
+    body = _AMINO_np = np.frombuffer(_AMINO, dtype=np.uint8)[rng.choice(20, size=length, p=_AMINO_FREQ)]
+    out = body.copy()
+    pos = int(rng.integers(60, 81))
+    while pos < length:
+        out[pos] = 10
+        pos += int(rng.integers(61, 82))
+    return out
+
+
+def long_lines(rng, length: int, words) -> np.ndarray:
+    """Text with very long lines (100 KiB - 4 MiB without a newline)."""
+    pool = _zipf_text(rng, min(length, 8 << 20) + 1, words, line=1 << 40)
+    reps = -(-length // pool.size)
+    buf = np.concatenate([np.roll(pool, -int(o)) for o in rng.integers(0, pool.size, size=reps)])[:length].copy() \
+        if reps > 1 else pool[:length].copy()
+    buf[buf == 10] = 32
+    pos = int(rng.integers(100 << 10, 4 << 20))
+    while pos < length:
+        buf[pos] = 10
+        pos += int(rng.integers(100 << 10, 4 << 20))
+    return buf
+
+
+def dotstar_input(length: int = 1 << 30, seed: int = 4, patterns_seed: int = 4, n_each: int = 1000,
+                  plant_every: int = 256 << 10):
+    """Half amino-acid lines, half long-line text (alternating 4 MiB stripes);
+    members of the pattern set planted about once per 256 KiB."""
+    rng = np.random.default_rng(seed * 7919 + 4)
+    stripe = 4 << 20
+    pool_len = min(length, 8 << 20) + stripe
+    am = amino_lines(rng, pool_len)
+    ll = long_lines(rng, pool_len, text_words())
+    buf = np.empty(length, dtype=np.uint8)
+    pos = 0
+    k = 0
+    while pos < length:
+        src = am if k % 2 == 0 else ll
+        n = min(stripe, length - pos)
+        o = int(rng.integers(0, src.size - n + 1))
+        buf[pos:pos + n] = src[o:o + n]
+        pos += n
+        k += 1
+    _, samplers = dotstar_protomata_patterns(n_each, patterns_seed)
+    _plant(rng, buf, samplers, plant_every)
+    return buf
+
+
+CONFIGS["dotstar"] = {
+    "patterns": lambda n=1000, seed=4: dotstar_protomata_patterns(n, seed)[0],
+    "input": lambda length=1 << 30, seed=4: dotstar_input(length, seed),
+    "pattern_kw": ("n",),
+    "input_kw": ("length",),
+    "len": 1 << 30,
+    "desc": "Dotstar/Protomata-like: 1,000 + 1,000 regexes over 1 GiB amino/long-line text (seed 4)",
+}
+
+
+# ---------------------------------------------------------------------------
+# config 5: 10k regexes (2,500 per family, seeds 51-54) over 8 GiB made of
+# four 2 GiB family inputs (seed 5)
+# ---------------------------------------------------------------------------
+def multi_patterns(n_each: int = 2500):
+    a = snort_patterns(n_each, 51)[0]
+    b = clamav_patterns(n_each // 2, 52)[0] + brill_patterns(n_each - n_each // 2, 52)[0]
+    c = dotstar_patterns(n_each, 53)[0]
+    d = protomata_patterns(n_each, 54)[0]
+    return a + b + c + d
+
+
+def multi_input(length: int = 8 << 30, seed: int = 5, part: int = None):
+    """The 8 GiB stream = snort-like | text | long-line/amino | amino, 2 GiB
+    each; `part` selects one quarter (generated independently, so a rank can
+    build only its own)."""
+    q = length // 4
+    gens = [lambda n: snort_input(n, seed=seed * 10 + 1, patterns_seed=51, n_patterns=2500),
+            lambda n: text_input(n, seed=seed * 10 + 2, patterns_seed=52, n_each=1250),
+            lambda n: dotstar_input(n, seed=seed * 10 + 3, patterns_seed=53, n_each=1250),
+            lambda n: amino_lines(np.random.default_rng(seed * 10 + 4), n)]
+    if part is not None:
+        return gens[part](q if part < 3 else length - 3 * q)
+    return np.concatenate([gens[i](q if i < 3 else length - 3 * q) for i in range(4)])
+
+
+CONFIGS["multi"] = {
+    "patterns": lambda n=2500: multi_patterns(n),
+    "input": lambda length=8 << 30, seed=5: multi_input(length, seed),
+    "pattern_kw": ("n",),
+    "input_kw": ("length",),
+    "len": 8 << 30,
+    "desc": "10k regexes (2,500 per family) over 8 GiB (seed 5)",
+}

@@ -36,7 +36,7 @@ struct RegexEmitter {
   std::ostringstream &os;
   const RegexIR &ir;
   int K;
-  int rloc;       // member index in the group
+  int rloc;       // cluster index in the group (names)
   int slot_base;  // first state slot of this regex in the group
   // CC / BDD-node caches by scope; scope 0 is shared by all regexes of the
   // group (their unguarded heads), deeper scopes are guard / loop bodies
@@ -338,18 +338,22 @@ struct RegexEmitter {
     }
   }
 
+  std::vector<int> out_member;  // group member index of each IR output
+
   void emit_output(int in) {
-    const Node &o = ir.nodes[ir.out];
-    if (o.op == Op::Zero) return;
-    std::string I = ind(in);
-    std::string R = nv(ir.out);
-    std::string m;
-    for (int i = 0; i < K; ++i) m += (i ? " | " : "") + ("(" + W(R, i) + " & c.cm[" + std::to_string(i) + "])");
-    os << I << "if (c.want_dense || __any_sync(RX_FULL, (" << m << ") != 0u)) {\n";
-    os << I << "  V<" << K << "> ov;\n";
-    for (int i = 0; i < K; ++i) os << I << "  ov.w[" << i << "] = " << W(R, i) << ";\n";
-    os << I << "  rx_emit<" << K << ">(c, " << rloc << ", ov);\n";
-    os << I << "}\n";
+    for (size_t k = 0; k < ir.outs.size(); ++k) {
+      const Node &o = ir.nodes[ir.outs[k]];
+      if (o.op == Op::Zero) continue;
+      std::string I = ind(in);
+      std::string R = nv(ir.outs[k]);
+      std::string m;
+      for (int i = 0; i < K; ++i) m += (i ? " | " : "") + ("(" + W(R, i) + " & c.cm[" + std::to_string(i) + "])");
+      os << I << "if (c.want_dense || __any_sync(RX_FULL, (" << m << ") != 0u)) {\n";
+      os << I << "  V<" << K << "> ov;\n";
+      for (int i = 0; i < K; ++i) os << I << "  ov.w[" << i << "] = " << W(R, i) << ";\n";
+      os << I << "  rx_emit<" << K << ">(c, " << out_member[k] << ", ov);\n";
+      os << I << "}\n";
+    }
   }
 
   // Two-phase emission: phase 1 holds every
@@ -392,7 +396,7 @@ struct RegexEmitter {
   // phase 1: returns the C expression "this regex needs phase 2"
   std::string emit_phase1() {
     classify();
-    os << "    // ---- regex member " << rloc << " (phase 1: unguarded head, guard tests)\n";
+    os << "    // ---- cluster " << rloc << " (phase 1: unguarded head, guard tests)\n";
     std::string need;
     for (int id : ir.blocks[0].nodes) {
       const Node &n = ir.nodes[id];
@@ -422,14 +426,16 @@ struct RegexEmitter {
     if (stateful_post) return "true";
     // the output must be produced even when no guard fires if it has an
     // unguarded contribution (e.g. an alternation with an unguarded branch)
-    if (has_guard && !zero_when_unfired(ir.out)) return "true";
+    if (has_guard)
+      for (int o : ir.outs)
+        if (!zero_when_unfired(o)) return "true";
     return has_guard ? need : "";
   }
 
   // phase 2 (inside `if (need)`)
   void emit_phase2() {
     if (!has_guard) return;
-    os << "    // ---- regex member " << rloc << " (phase 2: guarded bodies)\n";
+    os << "    // ---- cluster " << rloc << " (phase 2: guarded bodies)\n";
     push();
     for (int id : ir.blocks[0].nodes) {
       if (!post[id]) continue;
@@ -503,19 +509,22 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
     for (int i = 0; i < g.K; ++i) os << "    const u32 vmw" << i << " = c.vm[" << i << "];\n";
     std::vector<std::map<TabKey, std::string>> ccs(1);
     std::vector<std::map<std::vector<uint64_t>, std::string>> sets(1);
-    // one block per member: its unguarded head and guard tests (phase 1),
-    // then its guarded bodies (phase 2) if a guard fired
-    for (size_t m = 0; m < g.regexes.size(); ++m) {
-      const RegexIR &ir = cs.irs[g.regexes[m]];
-      RegexEmitter em(os, ir, g.K, (int)m, g.slot_base[m], ccs, sets);
+    // one block per factor cluster: its unguarded (shared) head and guard
+    // tests (phase 1), then its guarded bodies (phase 2) if a guard fired
+    for (size_t ci = 0; ci < g.clusters.size(); ++ci) {
+      const Cluster &cl = g.clusters[ci];
+      RegexEmitter em(os, cl.ir, g.K, (int)ci, cl.slot_base, ccs, sets);
+      em.out_member = cl.members;
       std::string run;
-      if ((g.always >> m) & 1u) {
+      if (cl.always) {
         run = "true";
       } else {
-        run = "((rmask >> " + std::to_string(m) + ") & 1u)";
-        if (ir.nslots > 0) {
+        uint32_t mm = 0;
+        for (int m : cl.members) mm |= 1u << m;
+        run = "(rmask & " + std::to_string(mm) + "u) != 0u";
+        if (cl.ir.nslots > 0) {
           std::string pend;
-          for (int sl = 0; sl < ir.nslots; ++sl) pend += (sl ? " | " : "") + em.st(sl);
+          for (int sl = 0; sl < cl.ir.nslots; ++sl) pend += (sl ? " | " : "") + em.st(sl);
           run += " || ((" + pend + ") != 0u)";
         }
       }
@@ -583,7 +592,7 @@ std::string emit_kernel_unit(CompiledSet &cs) {
   os << "    default: break;\n  }\n}\n";
   if (cs.use_pf)
     os << "\nextern \"C\" __global__ void __launch_bounds__(512, 1) rx_prefilter(const RxParams p) {\n"
-          "  rx_prefilter_run(p, RX_NG);\n}\n";
+          "  rx_prefilter_run(p, RX_NG, p.pf_tab_smem != 0);\n}\n";
   os << "\nextern \"C\" __global__ void __launch_bounds__(128) rx_fixup(const RxParams p) {\n"
         "  const int warp = threadIdx.x >> 5;\n"
         "  const int wpb = blockDim.x >> 5;\n"

@@ -179,11 +179,16 @@ struct RxParams {
   int accumulate;           // counts/digests are added to (else the host zeroed them)
   int lockstep;             // pass 1: one CTA barrier per window (warps of a group stay in step)
   // cross-regex prefilter (rx_prefilter below)
-  const u32 *pf_l1;         // [2048] bigram bitmap (last two bytes of every factor gram)
-  const u32 *pf_eoff;       // [65537] bigram -> entry range
-  const uint4 *pf_ent;      // {gram, mask, factor id, k}
-  const u32 *pf_fgoff;      // [nfactor+1] factor -> (group, member mask) range
-  const u32 *pf_fgent;      // {group, member mask}
+  // one table blob (rx_prefilter.cpp build_prefilter), u32 words:
+  //   [0,2048) l1 bigram bitmap | [2048,4096) rank: set bits before word i |
+  //   bsid[nb]: shapes indexed by each set bigram (shape = 3*(k-2) + d) |
+  //   htab[2 << hbits]: {gram, fid << 8 | shape << 1 | 1} | fgoff[nf+1] |
+  //   fgent[2*nfe]: {group, member mask}
+  const u32 *pf_tab;
+  u32 pf_words;             // blob size
+  u32 pf_o_ent, pf_o_fgoff, pf_o_fgent;  // word offsets: hash table, factor -> group ranges, pairs
+  u32 pf_hbits;             // log2 hash slots
+  int pf_tab_smem;          // the whole blob is staged in shared memory
   u32 *pf_gbits;            // [NG][ntiles]: bit b of word t = factor of the group in block 32t+b
   unsigned short *pf_blist; // [nblk][16]: hit count, then up to 15 factor ids (written for blocks with hits)
   i64 pf_ntiles;
@@ -616,26 +621,6 @@ DEV void rx_fixup_group(const RxParams &p, u64 *acc, u32 *sst) {
 #define RX_PF_BLK 1024
 #define RX_PF_TILE 32768
 
-DEV void rx_pf_hit(const RxParams &p, u32 *gt, u32 *blc, unsigned short *blf, u32 x, i64 q, i64 tile_lo) {
-  const u32 bg = x >> 16;
-  const u32 e1 = __ldg(&p.pf_eoff[bg + 1]);
-  for (u32 e = __ldg(&p.pf_eoff[bg]); e < e1; ++e) {
-    const uint4 en = __ldg(&p.pf_ent[e]);
-    if ((x & en.y) != en.x || q - (i64)en.w + 1 < p.avail_lo) continue;
-    const int b = (int)((q - tile_lo) >> 10);
-    const u32 fid = en.z;
-    bool dup = false;
-    const u32 n0 = *(volatile u32 *)&blc[b];
-    for (u32 j = 0; j < n0 && j < 15u; ++j)
-      if (*(volatile unsigned short *)&blf[b * 15 + j] == (unsigned short)fid) dup = true;
-    if (dup) continue;
-    const u32 slot = atomicAdd(&blc[b], 1u);
-    if (slot < 15u) blf[b * 15 + slot] = (unsigned short)fid;
-    const u32 f1 = __ldg(&p.pf_fgoff[fid + 1]);
-    for (u32 j = __ldg(&p.pf_fgoff[fid]); j < f1; ++j) atomicOr(&gt[__ldg(&p.pf_fgent[2 * j])], 1u << b);
-  }
-}
-
 DEV u32 rx_load_u32_slow(const RxParams &p, i64 pos) {
   u32 v = 0u;
   for (int j = 0; j < 4; ++j) {
@@ -645,14 +630,71 @@ DEV u32 rx_load_u32_slow(const RxParams &p, i64 pos) {
   return v;
 }
 
-DEV void rx_prefilter_run(const RxParams &p, int NG) {
+// x of position base + r (0 <= r < 20; 4 bytes ending there) from the words w0 (bytes base-4..base-1) .. w5 (base+16..base+19)
+DEV u32 rx_pf_x(u32 w0, u32 w1, u32 w2, u32 w3, u32 w4, u32 w5, int r) {
+  const int m = r >> 2, s = r & 3;
+  const u32 lo = m == 0 ? w0 : (m == 1 ? w1 : (m == 2 ? w2 : (m == 3 ? w3 : w4)));
+  const u32 hi = m == 0 ? w1 : (m == 1 ? w2 : (m == 2 ? w3 : (m == 3 ? w4 : w5)));
+  return s == 3 ? hi : __funnelshift_r(lo, hi, 8 * (s + 1));
+}
+
+// One queued hit of an index bigram: its end position (offset in the tile),
+// the 4 bytes ending there (xa) and the 4 bytes after them (xc); the gram
+// ends d = 0..3 bytes later and is x(d) = funnel(xa, xc, 8d).  It is recorded
+// in the block of the bigram's end (inside the gram, hence inside every
+// window frame that contains the gram).
+DEV void rx_pf_record(const RxParams &p, const u32 *T, u32 *gt, u32 *blc, unsigned short *blf, u32 fid, int b) {
+  bool dup = false;
+  const u32 n0 = *(volatile u32 *)&blc[b];
+  for (u32 j = 0; j < n0 && j < 15u; ++j)
+    if (*(volatile unsigned short *)&blf[b * 15 + j] == (unsigned short)fid) dup = true;
+  if (dup) return;
+  const u32 slot = atomicAdd(&blc[b], 1u);
+  if (slot < 15u) blf[b * 15 + slot] = (unsigned short)fid;
+  const u32 f1 = T[p.pf_o_fgoff + fid + 1];
+  for (u32 j = T[p.pf_o_fgoff + fid]; j < f1; ++j) atomicOr(&gt[T[p.pf_o_fgent + 2 * j]], 1u << b);
+}
+
+DEV void rx_pf_hit(const RxParams &p, const u32 *T, u32 *gt, u32 *blc, unsigned short *blf, u32 off, u32 xa,
+                   u32 xc, i64 tile_lo) {
+  const u32 bg = xa >> 16, wi = bg >> 5, bit = bg & 31u;
+  const u32 idx = T[2048 + wi] + __popc(T[wi] & ((1u << bit) - 1u));
+  u32 shapes = T[4096 + idx];
+  const int b = (int)(off >> 10);
+  const i64 q0 = tile_lo + off;
+  const u32 hmask = (1u << p.pf_hbits) - 1u;
+  const u32 *H = T + p.pf_o_ent;
+  while (shapes) {
+    const u32 sh = __ffs(shapes) - 1;
+    shapes &= shapes - 1u;
+    const u32 k = sh / 3u + 2u, d = sh - 3u * (k - 2u);
+    const u32 mask = k == 4u ? 0xffffffffu : (0xffffffffu << (8u * (4u - k)));
+    const u32 key = (d == 0u ? xa : __funnelshift_r(xa, xc, 8u * d)) & mask;
+    const i64 q = q0 + d;
+    if (q >= p.avail_hi || q - (i64)k + 1 < p.avail_lo) continue;
+    u32 h = ((key ^ (sh * 0x85EBCA6Bu)) * 0x9E3779B1u) >> (32u - p.pf_hbits);
+    for (;;) {
+      const u32 tag = H[2 * h + 1];
+      if (tag == 0u) break;
+      if (H[2 * h] == key && ((tag >> 1) & 127u) == sh) rx_pf_record(p, T, gt, blc, blf, tag >> 8, b);
+      h = (h + 1u) & hmask;
+    }
+  }
+}
+
+// smem: [tables (if they fit) | gt NG | blc 32 | blf 32 x 15 u16 | per-warp hit queues 32 x 3]
+DEV void rx_prefilter_run(const RxParams &p, int NG, bool tab_in_smem) {
   extern __shared__ __align__(16) u32 pf_smem[];
-  u32 *l1 = pf_smem;                 // 2048 words
-  u32 *blc = l1 + 2048;              // 32 hit counts
-  unsigned short *blf = reinterpret_cast<unsigned short *>(blc + 32);  // 32 x 15 factor ids
-  u32 *gt = blc + 32 + 240;          // NG words
   const int tid = threadIdx.x, nt = blockDim.x;
-  for (int i = tid; i < 2048; i += nt) l1[i] = __ldg(&p.pf_l1[i]);
+  const u32 tw = tab_in_smem ? ((p.pf_words + 3u) & ~3u) : 4096u;
+  u32 *tab = pf_smem;
+  for (u32 i = tid; i < tw && i < p.pf_words; i += nt) tab[i] = __ldg(&p.pf_tab[i]);
+  // l1 + rank are always staged; the rest is read through T
+  const u32 *T = tab_in_smem ? (const u32 *)tab : p.pf_tab;
+  u32 *gt = pf_smem + tw;
+  u32 *blc = gt + ((NG + 3) & ~3);
+  unsigned short *blf = reinterpret_cast<unsigned short *>(blc + 32);
+  u32 *wq = blc + 32 + 240 + 96 * (tid >> 5);  // per-warp hit queue: 32 x {off, xa, xc}
   const u32 lane = rx_lane();
   const i64 span = p.avail_hi - p.avail_lo;
   const i64 ntiles = (span + RX_PF_TILE - 1) / RX_PF_TILE;
@@ -663,27 +705,54 @@ DEV void rx_prefilter_run(const RxParams &p, int NG) {
     const i64 tile_lo = p.avail_lo + t * RX_PF_TILE;
     for (int j = 0; j < RX_PF_TILE / 16; j += nt) {
       const i64 base = tile_lo + (i64)(j + tid) * 16;
-      u32 w[5];
+      u32 w1, w2, w3, w4;
       if (p.pf_aligned && base + 16 <= p.avail_hi) {
         const uint4 v = __ldg(reinterpret_cast<const uint4 *>(p.in + base));
-        w[1] = v.x; w[2] = v.y; w[3] = v.z; w[4] = v.w;
+        w1 = v.x; w2 = v.y; w3 = v.z; w4 = v.w;
       } else {
-#pragma unroll
-        for (int m = 0; m < 4; ++m) w[m + 1] = rx_load_u32_slow(p, base + 4 * m);
+        w1 = rx_load_u32_slow(p, base);
+        w2 = rx_load_u32_slow(p, base + 4);
+        w3 = rx_load_u32_slow(p, base + 8);
+        w4 = rx_load_u32_slow(p, base + 12);
       }
-      w[0] = __shfl_up_sync(RX_FULL, w[4], 1);
-      if (lane == 0) w[0] = rx_load_u32_slow(p, base - 4);
+      u32 w0 = __shfl_up_sync(RX_FULL, w4, 1);
+      if (lane == 0) w0 = rx_load_u32_slow(p, base - 4);
+      u32 w5 = __shfl_down_sync(RX_FULL, w1, 1);
+      if (lane == 31) w5 = rx_load_u32_slow(p, base + 16);
+      // pass 1: bigram bitmap test of the 16 positions -> hit mask
+      u32 hm = 0u;
 #pragma unroll
-      for (int m = 0; m < 4; ++m) {
-#pragma unroll
-        for (int r = 0; r < 4; ++r) {
-          const u32 x = r == 3 ? w[m + 1] : __funnelshift_r(w[m], w[m + 1], 8 * (r + 1));
-          const u32 bg = x >> 16;
-          if ((l1[bg >> 5] >> (bg & 31)) & 1u) {
-            const i64 q = base + 4 * m + r;
-            if (q < p.avail_hi) rx_pf_hit(p, gt, blc, blf, x, q, tile_lo);
+      for (int r = 0; r < 16; ++r) {
+        const u32 x = rx_pf_x(w0, w1, w2, w3, w4, w5, r);
+        const u32 bg = x >> 16;
+        hm |= ((tab[bg >> 5] >> (bg & 31)) & 1u) << r;
+      }
+      const i64 rem = p.avail_hi - base;
+      if (rem < 16) hm &= rem <= 0 ? 0u : ((1u << rem) - 1u);
+      // pass 2: the warp's hits are compacted into a queue of 32 and checked
+      // one per lane (exact gram compare)
+      u32 qn = 0;
+      for (;;) {
+        const u32 bal = __ballot_sync(RX_FULL, hm != 0u);
+        if (bal) {
+          const u32 rk = __popc(bal & ((1u << lane) - 1u));
+          if (hm != 0u && qn + rk < 32u) {
+            const int r = __ffs(hm) - 1;
+            hm &= hm - 1u;
+            u32 *e = wq + 3 * (qn + rk);
+            e[0] = (u32)(base + r - tile_lo);
+            e[1] = rx_pf_x(w0, w1, w2, w3, w4, w5, r);
+            e[2] = rx_pf_x(w0, w1, w2, w3, w4, w5, r + 4);
           }
+          qn = qn + __popc(bal) < 32u ? qn + __popc(bal) : 32u;
         }
+        if (qn == 32u || (bal == 0u && qn > 0u)) {
+          __syncwarp();
+          if (lane < qn) rx_pf_hit(p, T, gt, blc, blf, wq[3 * lane], wq[3 * lane + 1], wq[3 * lane + 2], tile_lo);
+          __syncwarp();
+          qn = 0;
+        }
+        if (bal == 0u) break;
       }
     }
     __syncthreads();
@@ -785,9 +854,10 @@ template <class G> DEV void rx_run_segment_pf(const RxParams &p, int seg, u64 *a
       }
       if (c.lane < n) {
         const u32 fid = L[1 + c.lane];
-        const u32 f1 = __ldg(&p.pf_fgoff[fid + 1]);
-        for (u32 j = __ldg(&p.pf_fgoff[fid]); j < f1; ++j)
-          if (__ldg(&p.pf_fgent[2 * j]) == (u32)G::GID) mine |= __ldg(&p.pf_fgent[2 * j + 1]);
+        const u32 *fo = p.pf_tab + p.pf_o_fgoff, *fe = p.pf_tab + p.pf_o_fgent;
+        const u32 f1 = __ldg(&fo[fid + 1]);
+        for (u32 j = __ldg(&fo[fid]); j < f1; ++j)
+          if (__ldg(&fe[2 * j]) == (u32)G::GID) mine |= __ldg(&fe[2 * j + 1]);
       }
     }
     const u32 rmask = __reduce_or_sync(RX_FULL, mine);

@@ -89,7 +89,8 @@ struct RegexIR {
   std::vector<Node> nodes;
   std::vector<Block> blocks;  // blocks[0] = top level
   std::vector<ByteSet> sets;
-  int out = -1;               // result node (top level)
+  int out = -1;               // result node (top level) of a single-regex IR
+  std::vector<int> outs;      // result nodes of a cluster IR (one per member regex; outs[0] == out)
   int nslots = 0;
   int lb = 0, rb = 0;         // margins of the output (bits)
   int rb_state = 0;           // max rb over inputs of stateful sites (bits)
@@ -100,10 +101,18 @@ struct RegexIR {
 struct LowerOptions {
   int interval = 8;       // guard interval (instructions), <= 0: no guards
   bool rebalance = true;
+  // no zero-block guard inside the leading run of single-class items of an
+  // unanchored chain (with the prefilter the regex only runs where its
+  // factor occurs, and an unguarded head can be shared by a factor cluster)
+  bool lead_noguard = false;
 };
 
 // Lower one parsed regex to IR (non-empty, unanchored match ends).
 void lower_regex(const Ast &ast, const LowerOptions &opt, RegexIR &ir);
+// Lower several regexes into one IR with shared (hash-consed) nodes: a
+// factor cluster of a group is evaluated once per window (DESIGN.md
+// "Clusters").  ir.outs[i] is the result of asts[i].
+void lower_cluster(const std::vector<const Ast *> &asts, const LowerOptions &opt, RegexIR &ir);
 // Shift Rebalancing (Sec. 5.2): operand rewriting to a fixpoint + merging.
 void rebalance_regex(RegexIR &ir);
 // Compute margins, injection words and state slots.  Returns false if a
@@ -114,9 +123,17 @@ std::string dump_ir(const RegexIR &ir);
 // ----------------------------------------------------------------------------
 // Groups and program geometry
 // ----------------------------------------------------------------------------
+struct Cluster {
+  std::vector<int> members;  // member indices (into Group::regexes), in IR output order
+  RegexIR ir;                // shared IR of the members (lower_cluster)
+  int slot_base = 0;         // first state slot of the cluster in the group
+  bool always = false;       // members without a factor: runs in every window
+};
+
 struct Group {
   std::vector<int> regexes;  // global regex ids
   uint32_t always = 0;       // members without a prefilter factor (run in every window)
+  std::vector<Cluster> clusters;  // the group's code: members sharing a factor evaluated together
   int K = 1;                 // words per lane per window
   int Lw = 0, Rw = 0, Bw = 0;  // window: left halo words, right halo words, committed words (32K = Lw+Bw+Rw)
   int nslots = 0;
@@ -136,7 +153,9 @@ struct Factor {
 };
 struct Prefilter {
   int nfactor = 0;
-  std::vector<uint32_t> l1, e_off, ent, fg_off, fg_ent;
+  std::vector<uint32_t> blob;  // device table layout: see RxParams::pf_tab (rx_device.cuh)
+  uint32_t o_ent = 0, o_fgoff = 0, o_fgent = 0;  // o_ent: the gram hash table
+  uint32_t hbits = 0;                            // log2 of its slots
 };
 // Returns false if the regex has no usable factor (it then always runs).
 bool regex_factor(const Ast &a, Factor &f);
@@ -158,5 +177,9 @@ std::string emit_group_unit(CompiledSet &cs, int gi);
 std::string emit_kernel_unit(CompiledSet &cs);
 bool plan_groups(CompiledSet &cs, int group_size, int force_K, std::string &why);
 void build_prefilter(CompiledSet &cs);
+// Partition each group's members into clusters (same factor, or no factor)
+// and lower each cluster jointly; recomputes the group's state slots.
+bool build_clusters(CompiledSet &cs, const std::vector<const Ast *> &asts, const LowerOptions &opt,
+                    std::string &why);
 
 }  // namespace rx

@@ -198,6 +198,13 @@ struct Lowerer {
   // Concatenation items[j..] after a prefix whose (possibly empty) end
   // markers are P and whose non-empty end markers are N.
   int E_cat(const std::vector<Item> &items, size_t j, int P, int N, bool guarded = false) {
+    // leading run of single-class items of an unanchored chain: unguarded
+    // with opt.lead_noguard (LowerOptions)
+    size_t lead = 0;
+    if (opt.lead_noguard && j == 0 && is(P, Op::Ones) && loops.empty()) {
+      ByteSet tmp;
+      while (lead < items.size() && items[lead].mode == Item::Once && single_set(*items[lead].ast, tmp)) ++lead;
+    }
     for (; j < items.size(); ++j) {
       // Zero-block-skipping guard (Sec. 6): P is a zero-path
       // head -- if P is all-zero in a window, everything downstream in this
@@ -205,7 +212,7 @@ struct Lowerer {
       // head of the path (after its first shift+AND), then every `interval`
       // instructions.
       const bool head = !guarded && ir.nodes[P].op == Op::And;
-      if (opt.interval > 0 && loops.empty() && j > 0 && !is(P, Op::Ones) && !is(P, Op::Zero) &&
+      if (opt.interval > 0 && loops.empty() && j > 0 && j >= lead && !is(P, Op::Ones) && !is(P, Op::Zero) &&
           (head || since_guard >= (size_t)opt.interval) && ir.nodes[P].op != Op::CC) {
         Node g;
         g.op = Op::Guard;
@@ -297,7 +304,7 @@ struct Lowerer {
 
 }  // namespace
 
-void lower_regex(const Ast &ast, const LowerOptions &opt, RegexIR &ir) {
+void lower_cluster(const std::vector<const Ast *> &asts, const LowerOptions &opt, RegexIR &ir) {
   ir = RegexIR();
   ir.blocks.emplace_back();
   Lowerer L(ir, opt);
@@ -309,16 +316,22 @@ void lower_regex(const Ast &ast, const LowerOptions &opt, RegexIR &ir) {
   Node o;
   o.op = Op::Ones;
   L.ones = L.raw(o);
-  L.since_guard = 0;
   ir.n_instr = 0;
-  ir.out = L.E(ast, L.ones);
-  if (ir.out == L.ones) {
-    // a regex matching every position with a one-byte match of [\x00-\xff]
-    // cannot lower to Ones (Ones is 1 at padding too); E never returns Ones
-    // for a non-empty R, keep the guard anyway.
-    ir.out = L.CC([] { ByteSet s; s.range(0, 255); return s; }());
+  for (const Ast *a : asts) {
+    L.since_guard = 0;
+    int out = L.E(*a, L.ones);
+    if (out == L.ones) {
+      // a regex matching every position with a one-byte match of [\x00-\xff]
+      // cannot lower to Ones (Ones is 1 at padding too); E never returns Ones
+      // for a non-empty R, keep the guard anyway.
+      out = L.CC([] { ByteSet s; s.range(0, 255); return s; }());
+    }
+    ir.outs.push_back(out);
   }
+  ir.out = ir.outs.empty() ? L.zero : ir.outs[0];
 }
+
+void lower_regex(const Ast &ast, const LowerOptions &opt, RegexIR &ir) { lower_cluster({&ast}, opt, ir); }
 
 // ----------------------------------------------------------------------------
 // Margins: a window frame computes words [0, 32K); a
@@ -415,8 +428,11 @@ bool analyze_regex(RegexIR &ir, std::string &why) {
   int slot = 0;
   margins_block(ir, 0, slot);
   ir.nslots = slot;
-  ir.lb = ir.nodes[ir.out].lb;
-  ir.rb = ir.nodes[ir.out].rb;
+  ir.lb = ir.rb = 0;
+  for (int o : ir.outs) {
+    ir.lb = std::max(ir.lb, ir.nodes[o].lb);
+    ir.rb = std::max(ir.rb, ir.nodes[o].rb);
+  }
   (void)why;
   return true;
 }
@@ -526,6 +542,54 @@ bool plan_groups(CompiledSet &cs, int group_size, int force_K, std::string &why)
     gr.Lw = L;
     gr.Rw = R;
     gr.Bw = 32 * K - L - R;
+  }
+  return true;
+}
+
+// Factor clusters: inside a group, members with the
+// same prefilter factor are woken by the same hits, so they are lowered
+// together and their common prefix (shared CCs, shifts and ANDs up to the
+// first zero-block guard) is computed once per window; members without a
+// factor form one cluster that runs in every window.
+bool build_clusters(CompiledSet &cs, const std::vector<const Ast *> &asts, const LowerOptions &opt,
+                    std::string &why) {
+  for (auto &g : cs.groups) {
+    g.clusters.clear();
+    std::map<int, int> by_factor;  // factor id (-1 = none) -> cluster
+    for (size_t m = 0; m < g.regexes.size(); ++m) {
+      const int r = g.regexes[m];
+      const int f = cs.factor_of.empty() ? -1 : cs.factor_of[r];
+      auto it = by_factor.find(f);
+      int ci;
+      if (it == by_factor.end()) {
+        ci = (int)g.clusters.size();
+        by_factor[f] = ci;
+        g.clusters.emplace_back();
+        g.clusters.back().always = f < 0;
+      } else {
+        ci = it->second;
+      }
+      g.clusters[ci].members.push_back((int)m);
+    }
+    int L = 0, R = 0;
+    g.nslots = 0;
+    for (auto &c : g.clusters) {
+      std::vector<const Ast *> as;
+      for (int m : c.members) as.push_back(asts[g.regexes[m]]);
+      LowerOptions co = opt;
+      co.lead_noguard = opt.lead_noguard && !c.always;
+      lower_cluster(as, co, c.ir);
+      if (opt.rebalance) rebalance_regex(c.ir);
+      if (!analyze_regex(c.ir, why)) return false;
+      c.slot_base = g.nslots;
+      g.nslots += c.ir.nslots;
+      L = std::max(L, (c.ir.lb + 31) / 32);
+      R = std::max(R, (std::max(c.ir.rb, c.ir.rb_state) + 31) / 32);
+    }
+    if (L > g.Lw || R > g.Rw) {
+      why = "cluster margins exceed the group window";
+      return false;
+    }
   }
   return true;
 }

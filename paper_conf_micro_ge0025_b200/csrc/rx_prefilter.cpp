@@ -223,32 +223,69 @@ bool regex_factor(const Ast &a, Factor &f) {
   return true;
 }
 
-// Device tables of the prefilter (layout documented in rx_device.cuh,
-// rx_prefilter kernel):
-//   l1[2048]        bitmap over the 65,536 bigrams = last two bytes of a gram
-//   e_off[65537]    CSR over that bigram -> entries
-//   ent[4*n]        {gram, mask, factor id, k}
-//   fg_off[nf+1]    CSR over factors -> (group, member mask) pairs
-//   fg_ent[2*m]
+// Device tables of the prefilter, one u32 blob (layout documented at
+// RxParams::pf_tab in rx_device.cuh):
+//   l1[2048]     bitmap over the 65,536 bigrams: each gram's index bigram
+//                (its rarest byte pair under the model)
+//   rank[2048]   set bits of l1 before word i (compact index of a set bigram)
+//   bsid[nb]     per set bigram: mask of the gram shapes indexed by it; shape
+//                s = 3*(k-2) + d (k = gram length, d = gram bytes after the
+//                index bigram)
+//   htab[2*HS]   open-addressing hash set of (gram, shape) -> factor:
+//                {gram, factor << 8 | shape << 1 | 1}; empty slots are 0
+//   fgoff[nf+1]  per factor: its range of (group, member mask) pairs
+//   fgent[2*m]
+uint32_t pf_hash(uint32_t gram, uint32_t shape) { return (gram ^ (shape * 0x85EBCA6Bu)) * 0x9E3779B1u; }
+
 void build_prefilter(CompiledSet &cs) {
   Prefilter &pf = cs.pf;
   pf = Prefilter();
   const int nf = (int)cs.factors.size();
   pf.nfactor = nf;
-  pf.l1.assign(2048, 0u);
-  std::vector<std::vector<uint32_t>> by_bg(65536);
+  std::vector<uint32_t> l1(2048, 0u);
+  std::map<uint32_t, uint32_t> sids;  // index bigram -> shape mask
+  struct E { uint32_t gram, shape, fid; };
+  std::vector<E> ents;
+  const Model &mdl = model();
   for (int f = 0; f < nf; ++f)
     for (auto &g : cs.factors[f].grams) {
-      const uint32_t bg = g.gram >> 16;
-      pf.l1[bg >> 5] |= 1u << (bg & 31);
-      by_bg[bg].insert(by_bg[bg].end(), {g.gram, g.mask, (uint32_t)f, (uint32_t)g.k});
+      int best_d = 0;
+      double best_p = 2.0;
+      for (int d = 0; d + 2 <= g.k; ++d) {
+        const int b1 = (g.gram >> (8 * (2 - d))) & 255, b2 = (g.gram >> (8 * (3 - d))) & 255;
+        const double pp = mdl.p[b1] * mdl.p[b2];
+        if (pp < best_p) {
+          best_p = pp;
+          best_d = d;
+        }
+      }
+      const uint32_t bg = (g.gram >> (8 * (2 - best_d))) & 0xffffu;
+      const uint32_t shape = 3u * (uint32_t)(g.k - 2) + (uint32_t)best_d;
+      l1[bg >> 5] |= 1u << (bg & 31);
+      sids[bg] |= 1u << shape;
+      ents.push_back(E{g.gram, shape, (uint32_t)f});
     }
-  pf.e_off.assign(65537, 0u);
-  for (int b = 0; b < 65536; ++b) {
-    pf.e_off[b] = (uint32_t)(pf.ent.size() / 4);
-    pf.ent.insert(pf.ent.end(), by_bg[b].begin(), by_bg[b].end());
+  std::vector<uint32_t> &B = pf.blob;
+  B = l1;
+  uint32_t run = 0;
+  for (int i = 0; i < 2048; ++i) {
+    B.push_back(run);
+    run += (uint32_t)__builtin_popcount(l1[i]);
   }
-  pf.e_off[65536] = (uint32_t)(pf.ent.size() / 4);
+  for (auto &kv : sids) B.push_back(kv.second);  // ascending bigram = ascending rank
+  uint32_t hs = 64;
+  while (hs < 2 * ents.size()) hs <<= 1;
+  pf.hbits = 0;
+  while ((1u << pf.hbits) < hs) ++pf.hbits;
+  pf.o_ent = (uint32_t)B.size();
+  std::vector<uint32_t> ht(2 * hs, 0u);
+  for (auto &e : ents) {
+    uint32_t h = pf_hash(e.gram, e.shape) >> (32 - pf.hbits);
+    while (ht[2 * h + 1] != 0u) h = (h + 1) & (hs - 1);
+    ht[2 * h] = e.gram;
+    ht[2 * h + 1] = (e.fid << 8) | (e.shape << 1) | 1u;
+  }
+  B.insert(B.end(), ht.begin(), ht.end());
   // factor -> groups
   std::vector<std::map<int, uint32_t>> fg(nf);
   for (int gi = 0; gi < (int)cs.groups.size(); ++gi) {
@@ -258,12 +295,15 @@ void build_prefilter(CompiledSet &cs) {
       if (f >= 0) fg[f][gi] |= 1u << m;
     }
   }
-  pf.fg_off.assign(nf + 1, 0u);
+  pf.o_fgoff = (uint32_t)B.size();
+  std::vector<uint32_t> fge;
   for (int f = 0; f < nf; ++f) {
-    pf.fg_off[f] = (uint32_t)(pf.fg_ent.size() / 2);
-    for (auto &kv : fg[f]) pf.fg_ent.insert(pf.fg_ent.end(), {(uint32_t)kv.first, kv.second});
+    B.push_back((uint32_t)(fge.size() / 2));
+    for (auto &kv : fg[f]) fge.insert(fge.end(), {(uint32_t)kv.first, kv.second});
   }
-  pf.fg_off[nf] = (uint32_t)(pf.fg_ent.size() / 2);
+  B.push_back((uint32_t)(fge.size() / 2));
+  pf.o_fgent = (uint32_t)B.size();
+  B.insert(B.end(), fge.begin(), fge.end());
 }
 
 }  // namespace rx

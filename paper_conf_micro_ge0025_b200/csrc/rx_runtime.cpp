@@ -188,7 +188,6 @@ struct RxModule {
   CUfunction pass1 = nullptr, fixup = nullptr, prefilter = nullptr;
   // prefilter tables on the device (uploaded at load)
   void *pf_mem = nullptr;
-  const void *pf_l1 = nullptr, *pf_eoff = nullptr, *pf_ent = nullptr, *pf_fgoff = nullptr, *pf_fgent = nullptr;
 };
 
 struct rx_program {
@@ -252,6 +251,7 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
   p->n_regex = n_patterns;
   p->cs.irs.resize(n_patterns);
   p->cs.factor_of.assign(n_patterns, -1);
+  std::vector<rx::AstP> asts(n_patterns);
   const bool use_pf = !(o.flags & RX_F_NO_PREFILTER);
   std::map<std::vector<uint32_t>, int> factor_ix;
   for (uint32_t i = 0; i < n_patterns; ++i) {
@@ -293,13 +293,18 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
       }
       p->cs.factor_of[i] = fid;
     }
-    rx::lower_regex(*ast, lo, p->cs.irs[i]);
+    {
+      rx::LowerOptions ro = lo;
+      ro.lead_noguard = use_pf && p->cs.factor_of[i] >= 0;
+      rx::lower_regex(*ast, ro, p->cs.irs[i]);
+    }
     if (lo.rebalance) rx::rebalance_regex(p->cs.irs[i]);
     std::string why;
     if (!rx::analyze_regex(p->cs.irs[i], why)) {
       delete p;
       return fail(RX_EUNSUPPORTED, why);
     }
+    asts[i] = std::move(ast);
   }
   std::string why;
   if (!rx::plan_groups(p->cs, (int)o.group_size, (int)o.words_per_lane, why)) {
@@ -312,6 +317,16 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
     return fail(RX_ETOOBIG, why);
   }
   p->cs.use_pf = !p->cs.factors.empty();
+  {
+    std::vector<const rx::Ast *> ap;
+    for (auto &a : asts) ap.push_back(a.get());
+    rx::LowerOptions co = lo;
+    co.lead_noguard = p->cs.use_pf;
+    if (!rx::build_clusters(p->cs, ap, co, why)) {
+      delete p;
+      return fail(RX_EUNSUPPORTED, why);
+    }
+  }
   if (p->cs.use_pf) rx::build_prefilter(p->cs);
   // one relocatable NVRTC unit per group + the kernel unit, compiled in
   // parallel and linked into one module by nvJitLink
@@ -418,7 +433,11 @@ struct RxParamsHost {  // must mirror RxParams in rx_device.cuh
   int mode;
   int accumulate;
   int lockstep;
-  const void *pf_l1, *pf_eoff, *pf_ent, *pf_fgoff, *pf_fgent;
+  const unsigned int *pf_tab;
+  unsigned int pf_words;
+  unsigned int pf_o_ent, pf_o_fgoff, pf_o_fgent;
+  unsigned int pf_hbits;
+  int pf_tab_smem;
   unsigned int *pf_gbits;
   unsigned short *pf_blist;
   long long pf_ntiles;
@@ -462,23 +481,9 @@ rx_status ensure_loaded(rx_program *p, int &device) {
       if (d.ModuleGetFunction(&m.prefilter, m.mod, "rx_prefilter") != CUDA_SUCCESS)
         return fail(RX_ECUDA, "rx_prefilter symbol missing");
       const rx::Prefilter &pf = p->cs.pf;
-      const std::vector<uint32_t> *parts[] = {&pf.l1, &pf.e_off, &pf.ent, &pf.fg_off, &pf.fg_ent};
-      size_t off[5], total = 0;
-      for (int i = 0; i < 5; ++i) {
-        off[i] = total;
-        total += (4 * parts[i]->size() + 255) & ~(size_t)255;
-      }
-      if (cudaMalloc(&m.pf_mem, total + 256) != cudaSuccess) return fail(RX_ENOMEM, "prefilter tables");
-      for (int i = 0; i < 5; ++i)
-        if (!parts[i]->empty() &&
-            cudaMemcpy((char *)m.pf_mem + off[i], parts[i]->data(), 4 * parts[i]->size(), cudaMemcpyHostToDevice) !=
-                cudaSuccess)
-          return fail(RX_ECUDA, "prefilter table upload");
-      m.pf_l1 = (char *)m.pf_mem + off[0];
-      m.pf_eoff = (char *)m.pf_mem + off[1];
-      m.pf_ent = (char *)m.pf_mem + off[2];
-      m.pf_fgoff = (char *)m.pf_mem + off[3];
-      m.pf_fgent = (char *)m.pf_mem + off[4];
+      if (cudaMalloc(&m.pf_mem, 4 * pf.blob.size() + 16) != cudaSuccess) return fail(RX_ENOMEM, "prefilter tables");
+      if (cudaMemcpy(m.pf_mem, pf.blob.data(), 4 * pf.blob.size(), cudaMemcpyHostToDevice) != cudaSuccess)
+        return fail(RX_ECUDA, "prefilter table upload");
     }
     m.device = device;
   }
@@ -498,7 +503,8 @@ rx_status launch(RxModule &m, CUfunction f, long long blocks, int warps_per_bloc
   const size_t wpb = (size_t)warps_per_block;
   size_t bytes = wpb * 3 * m.nr_max * 8 + (((wpb * 4 * m.ns_max) + 3) & ~(size_t)3) * 4;
   if (f == m.pass1) bytes += wpb * 4096 + wpb * 16;
-  if (f == m.prefilter) bytes = 4 * (2048 + 32 + 240 + (size_t)(m.g_end - m.g_begin));
+  if (f == m.prefilter)
+    bytes = 4 * ((prm.pf_tab_smem ? ((prm.pf_words + 3) & ~3u) : 4096u) + (((m.g_end - m.g_begin) + 3) & ~3) + 32 + 240 + 96 * (size_t)warps_per_block);
   unsigned smem = (unsigned)bytes;
   if (smem > 48 * 1024) d.FuncSetAttribute(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)smem);
   RxParamsHost local = prm;
@@ -609,11 +615,13 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
       const size_t bl_bytes = (size_t)ntiles * 32 * 32;
       if (cudaMallocAsync(&pf_scratch, gb_bytes + bl_bytes + 256, stream) != cudaSuccess)
         return fail(RX_ENOMEM, "prefilter scratch");
-      prm.pf_l1 = m.pf_l1;
-      prm.pf_eoff = m.pf_eoff;
-      prm.pf_ent = m.pf_ent;
-      prm.pf_fgoff = m.pf_fgoff;
-      prm.pf_fgent = m.pf_fgent;
+      prm.pf_tab = (const unsigned int *)m.pf_mem;
+      prm.pf_words = (unsigned int)p->cs.pf.blob.size();
+      prm.pf_o_ent = p->cs.pf.o_ent;
+      prm.pf_o_fgoff = p->cs.pf.o_fgoff;
+      prm.pf_o_fgent = p->cs.pf.o_fgent;
+      prm.pf_hbits = p->cs.pf.hbits;
+      prm.pf_tab_smem = 4ull * prm.pf_words <= 160 * 1024 ? 1 : 0;
       prm.pf_gbits = (unsigned int *)pf_scratch;
       prm.pf_blist = (unsigned short *)((char *)pf_scratch + ((gb_bytes + 255) & ~(size_t)255));
       prm.pf_ntiles = ntiles;

@@ -72,3 +72,25 @@ def test_snort_like_patterns_all_compile_to_ir():
         assert oracle.check(p)[0] == 0
     # a slice through the full pipeline including NVRTC
     rx.Program(pats[:24])
+
+
+def _struct_fields(src, name):
+    body = re.search(r"struct " + name + r" \{(.*?)\n\};", src, re.S).group(1)
+    body = re.sub(r"//[^\n]*", "", body)
+    names = []
+    for decl in body.split(";"):
+        decl = decl.strip()
+        if not decl:
+            continue
+        ty, rest = re.match(r"((?:const\s+)?(?:unsigned\s+)?(?:long\s+long|[A-Za-z0-9_]+)\s*\**)\s*(.*)", decl,
+                            re.S).groups()
+        for v in rest.split(","):
+            names.append(v.strip().lstrip("*"))
+    return names
+
+
+def test_kernel_param_struct_mirrors_match():
+    dev = open(os.path.join(ROOT, "paper_conf_micro_ge0025_b200", "csrc", "rx_device.cuh")).read()
+    host = open(os.path.join(ROOT, "paper_conf_micro_ge0025_b200", "csrc", "rx_runtime.cpp")).read()
+    a, b = _struct_fields(dev, "RxParams"), _struct_fields(host, "RxParamsHost")
+    assert a == b, (a, b)
