@@ -194,6 +194,8 @@ struct RxParams {
   i64 pf_ntiles;
   int pf_on;
   int pf_aligned;           // in + avail_lo is 16-byte aligned
+  u64 *stats;               // nullable: debug counters (RX_STATS=1), see rx_run_segment_pf
+  int dbg;                  // timing experiments only (RX_DBG): 1 = skip every window, 2 = no body
 };
 
 template <int K> DEV void rx_load_window(const RxParams &p, Ctx<K> &c, u32 (&pl)[8][K], i64 fword) {
@@ -821,8 +823,19 @@ template <class G> DEV void rx_run_segment_pf(const RxParams &p, int seg, u64 *a
     i64 t0;
     frame_blocks(w_end - 1, t0, bmax);
   }
+  // lockstep (p.lockstep): the CTA's warps step through window i together
+  // (one barrier per step) so that they fetch the group's code together;
+  // otherwise each warp jumps to its next window with a factor hit
+  const bool lockstep = p.lockstep != 0;
   i64 w = w_begin;
-  while (w < w_end) {
+  int step = 0;
+  while (lockstep ? step < p.sw : w < w_end) {
+    if (lockstep) {
+      if (step > 0) __syncthreads();
+      w = w_begin + step;
+      ++step;
+      if (w >= w_end) continue;
+    }
     i64 b0, b1;
     frame_blocks(w, b0, b1);
     bool pend = false;
@@ -831,8 +844,15 @@ template <class G> DEV void rx_run_segment_pf(const RxParams &p, int seg, u64 *a
       for (int s = (int)c.lane; s < NS; s += 32) any = any || st[s] != 0u;
       pend = __any_sync(RX_FULL, any);
     }
+    if (p.stats && c.lane == 0) atomicAdd(&p.stats[3], 1ull);  // [3] window visits (checks)
+    if (p.dbg == 1) {
+      if (lockstep) continue;
+      ++w;
+      continue;
+    }
     if (!pend && G::ALWAYS == 0u) {
-      const i64 b = rx_pf_next(gb, b0, bmax, c.lane);
+      const i64 b = rx_pf_next(gb, b0, lockstep ? b1 : bmax, c.lane);
+      if (lockstep && b > b1) continue;
       if (b > b1) {
         if (b > bmax) break;
         // the first window whose frame reaches block b
@@ -861,6 +881,12 @@ template <class G> DEV void rx_run_segment_pf(const RxParams &p, int seg, u64 *a
       }
     }
     const u32 rmask = __reduce_or_sync(RX_FULL, mine);
+    if (p.stats && c.lane == 0) {
+      // [0] active windows [1] of them only for carried state [2] members hit
+      atomicAdd(&p.stats[0], 1ull);
+      if (rmask == 0u) atomicAdd(&p.stats[1], 1ull);
+      atomicAdd(&p.stats[2], (u64)__popc(rmask));
+    }
     const i64 cstart = w * Bw;
     const i64 fword = cstart - Lw;
     c.cw = (u32)((len_words - cstart) < Bw ? (len_words - cstart) : Bw);
@@ -869,13 +895,18 @@ template <class G> DEV void rx_run_segment_pf(const RxParams &p, int seg, u64 *a
     rx_unpack<K>(p, ir, c, xr, pl, fword);
     rx_commit_mask(p, ir, c, Lw, fword);
     if (NS > 0) rx_state_zero(nst, NS, c.lane);
-    G::body(c, pl, st, nst, rmask);
+    if (p.dbg == 2) {
+      if (c.lane == 0 && (pl[0][0] ^ pl[7][K - 1]) == 0x12345u) atomicAdd(p.status, 0u);  // keep the loads
+    } else {
+      G::body(c, pl, st, nst, rmask);
+    }
     u32 *t = st;
     st = nst;
     nst = t;
     __syncwarp();
-    ++w;
+    if (!lockstep) ++w;
   }
+  if (lockstep && step > 0) __syncthreads();
   if (!live) return;
   if (NS > 0) {
     u32 *dst = p.seg_state + ((i64)seg * G::NG + G::GID) * G::NSMAX;

@@ -15,6 +15,7 @@
 // part; concatenation tracks P (prefix may be empty) and N (non-empty).
 #include <algorithm>
 #include <cassert>
+#include <cstdlib>
 #include <cstring>
 #include <functional>
 #include <map>
@@ -496,7 +497,12 @@ bool plan_groups(CompiledSet &cs, int group_size, int force_K, std::string &why)
   size_t total_instr = 0;
   for (auto &r : cs.irs) total_instr += r.n_instr;
   if (group_size <= 0 || group_size > 32) group_size = 32;  // member masks are 32-bit
-  const size_t max_instr = 1500;  // bounds one NVRTC unit (compile time) and the group's code size
+  // bounds one NVRTC unit (compile time) and the group's code size (the
+  // SM's instruction caches hold one group's program); RX_GROUP_INSTR
+  // overrides (experiments)
+  size_t max_instr = 1500;
+  if (const char *e = getenv("RX_GROUP_INSTR"))
+    if (atoi(e) > 0) max_instr = (size_t)atoi(e);
   cs.groups.clear();
   Group g;
   size_t gi = 0;

@@ -443,6 +443,8 @@ struct RxParamsHost {  // must mirror RxParams in rx_device.cuh
   long long pf_ntiles;
   int pf_on;
   int pf_aligned;
+  unsigned long long *stats;
+  int dbg;
 };
 
 rx_status ensure_loaded(rx_program *p, int &device) {
@@ -627,11 +629,31 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
       prm.pf_ntiles = ntiles;
       prm.pf_on = 1;
       prm.pf_aligned = (((uintptr_t)(d_input - halo_left)) & 15) == 0 ? 1 : 0;
-      prm.lockstep = 0;
+      {
+        const char *e = getenv("RX_PF_LOCKSTEP");  // experiment knob
+        prm.lockstep = (e && *e == '1') ? 1 : 0;
+      }
       s = launch(m, m.prefilter, std::min<long long>(ntiles, 148LL * 4), 16, prm, stream);
       if (s != RX_OK) return s;
     }
+    unsigned long long *stats = nullptr;
+    const char *se = getenv("RX_STATS");
+    if (se && *se == '1' && cudaMalloc((void **)&stats, 64) == cudaSuccess) cudaMemsetAsync(stats, 0, 64, stream);
+    prm.stats = stats;
+    {
+      const char *de = getenv("RX_DBG");  // timing experiments only: results are wrong when set
+      prm.dbg = (de && *de) ? atoi(de) : 0;
+    }
     s = launch(m, m.pass1, cpg * mg, kPass1Warps, prm, stream);
+    prm.stats = nullptr;
+    if (stats) {
+      unsigned long long h[8];
+      cudaMemcpyAsync(h, stats, 64, cudaMemcpyDeviceToHost, stream);
+      cudaStreamSynchronize(stream);
+      fprintf(stderr, "[rx stats] groups=%d window_checks=%llu active=%llu state_only=%llu member_hits=%llu\n", mg,
+              h[3], h[0], h[1], h[2]);
+      cudaFree(stats);
+    }
     if (pf_scratch) cudaFreeAsync(pf_scratch, stream);
     prm.pf_on = 0;
     if (s != RX_OK) return s;

@@ -1,0 +1,129 @@
+"""Host-side multi-GPU protocol (paper_conf_micro_ge0025_b200/parallel.py) on
+CPU with the gloo backend, world sizes 2 and 3.
+
+The GPU matching is replaced by a small exact model of a chunk's boundary
+state so that the protocol -- speculative zero-state match, sequential state
+resolution by broadcast, rematch only where the true incoming state differs,
+all-reduce of per-regex counts -- is checked end to end across processes.
+The model: the "regex" counts positions where the running count of byte 'a'
+since the last 'z' is odd; the boundary state is that parity (a carried
+state in the sense of DESIGN.md "Forwarded state").
+"""
+import os
+import socket
+
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from paper_conf_micro_ge0025_b200 import parallel
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def model_match(data: bytes, state_in: int):
+    """(count, state_out) of the toy carried-state program."""
+    par = state_in
+    n = 0
+    for b in data:
+        if b == ord("z"):
+            par = 0
+        elif b == ord("a"):
+            par ^= 1
+        n += par
+    return n, par
+
+
+class FakeProg:
+    """Stands in for parallel.ChunkMatcher's Program (CPU tensors)."""
+
+    def __init__(self, data: bytes):
+        self.data = data
+        self.boundary_bytes = 4
+        self.calls = []
+
+    def match_chunk(self, buf, length, halo_left, halo_right, global_offset, state_in=None, state_out=None,
+                    out=None):
+        s_in = 0 if state_in is None else int(state_in[0])
+        chunk = self.data[global_offset:global_offset + length]
+        n, s_out = model_match(chunk, s_in)
+        out["counts"][0] = n
+        state_out[0] = s_out
+        self.calls.append(("match", s_in))
+
+    def rematch_chunk(self, buf, length, halo_left, halo_right, global_offset, assumed, true, state_out, out):
+        chunk = self.data[global_offset:global_offset + length]
+        n_old, _ = model_match(chunk, int(assumed[0]))
+        n_new, s_out = model_match(chunk, int(true[0]))
+        out["counts"][0] += n_new - n_old
+        state_out[0] = s_out
+        self.calls.append(("rematch", int(true[0])))
+
+
+def _worker(rank, world, port, data, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        prog = FakeProg(data)
+        cm = parallel.ChunkMatcher(prog, torch.device("cpu"), dist=dist)
+        a, b = parallel.chunk_bounds(len(data), world, rank)
+        out = {"counts": torch.zeros(1, dtype=torch.int64), "digests": None}
+        reruns = cm.match_chunk(None, b - a, 0, 0, a, rank, world, out)
+        q.put((rank, int(out["counts"][0]), reruns, prog.calls))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_chunked_protocol_equals_whole_stream(world):
+    rng = torch.Generator().manual_seed(world)
+    alphabet = b"aazbc"
+    data = bytes(alphabet[i] for i in torch.randint(0, len(alphabet), (3000,), generator=rng).tolist())
+    data = data[:1000] + b"a" + b"b" * 999 + data[2000:]  # a parity carried across a chunk boundary
+    whole, _ = model_match(data, 0)
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, data, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=120) for _ in procs]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    res.sort()
+    # every rank holds the all-reduced total == the whole-stream count
+    assert all(r[1] == whole for r in res), (whole, res)
+    # rank r re-ran iff its true incoming state was not the assumed zero
+    for rank, _, reruns, calls in res:
+        a, _ = parallel.chunk_bounds(len(data), world, rank)
+        _, true_in = model_match(data[:a], 0)
+        assert reruns == (1 if rank > 0 and true_in != 0 else 0)
+        if reruns:
+            assert calls[-1] == ("rematch", true_in)
+
+
+def test_shard_patterns_is_a_balanced_partition():
+    costs = [float(c) for c in [5, 1, 9, 3, 3, 7, 2, 8, 1, 4]]
+    for world in (1, 2, 3, 4):
+        shards = [parallel.shard_patterns(len(costs), world, r, costs) for r in range(world)]
+        flat = sorted(i for s in shards for i in s)
+        assert flat == list(range(len(costs)))
+        loads = [sum(costs[i] for i in s) for s in shards]
+        assert max(loads) - min(loads) <= max(costs)
+
+
+def test_chunk_bounds_cover_the_stream():
+    for n in (0, 1, 7, 1000):
+        for world in (1, 2, 3, 8):
+            cuts = [parallel.chunk_bounds(n, world, r) for r in range(world)]
+            assert cuts[0][0] == 0 and cuts[-1][1] == n
+            assert all(cuts[i][1] == cuts[i + 1][0] for i in range(world - 1))
