@@ -109,8 +109,18 @@ typedef struct {
   uint64_t *d_digests;    /* nullable: u64[2*n_regex]: sum splitmix64(p), sum splitmix64(p^0x9E3779B97F4A7C15) */
   uint32_t *d_bitstreams; /* nullable: u32[n_regex * pitch_words], LSB-first (bit p of word p/32); bits >= len are 0 */
   uint64_t pitch_words;   /* >= ceil(len/32) when d_bitstreams != NULL */
-  uint32_t *d_status;     /* nullable: u32 device flags, bit0 = iteration cap hit (result not exact) */
-  uint32_t reserved[4];
+  uint32_t *d_status;     /* nullable: u32 device flags, bit0 = iteration cap hit (result not exact),
+                             bit2 = a fix-up run lost a match the speculative run listed (never expected:
+                             match sets are monotone in the incoming state) */
+  /* Compacted match list ("match positions"): one entry per set bit of
+   * every S_r, {regex id, global position}, in no particular order.  Both
+   * nullable; d_matches requires d_match_total.  *d_match_total receives the
+   * true number of matches (zeroed unless accumulating); entries beyond
+   * match_cap are dropped, so a caller seeing total > cap re-runs with a
+   * larger list.  With d_match_total alone the total is counted only. */
+  rx_match_t *d_matches;
+  uint64_t match_cap;
+  uint64_t *d_match_total;
 } rx_output;
 
 /* Match the whole input d_input[0..len).  Asynchronous on `stream`
@@ -135,6 +145,15 @@ rx_status rx_match_chunk(const rx_program *p, const uint8_t *d_input, uint64_t l
 rx_status rx_rematch_chunk(const rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo_left,
                            uint64_t halo_right, uint64_t global_offset, const void *d_state_assumed,
                            const void *d_state_true, void *d_state_out, void *stream, const rx_output *out);
+
+/* Per-kernel device timing (for roofline reporting): when on, every launch
+ * of the program is bracketed by CUDA events on its stream.  rx_kernel_times
+ * waits for the recorded events and writes the accumulated milliseconds and
+ * launch counts of the three kernels, ms[0..2] / launches[0..2] = prefilter,
+ * pass 1 (the fused interleaved kernel), fix-up; reset != 0 zeroes them. */
+rx_status rx_set_profiling(rx_program *p, int on);
+rx_status rx_kernel_times(rx_program *p, double *ms /* [3], nullable */, uint64_t *launches /* [3], nullable */,
+                          int reset);
 
 /* Last error message of this thread (static storage). */
 const char *rx_last_error(void);

@@ -50,6 +50,8 @@ def _load():
             lib.orc_free.argtypes = [vp]
             lib.orc_num_states.argtypes = [vp]
             lib.orc_nullable.argtypes = [vp]
+            lib.orc_max_len.argtypes = [vp]
+            lib.orc_max_len.restype = ctypes.c_int64
             lib.orc_run.argtypes = [vp, vp, u64, ctypes.c_int, ctypes.c_int, vp, vp, u64,
                                     ctypes.POINTER(u64), ctypes.POINTER(u64)]
             lib.orc_run.restype = u64
@@ -107,6 +109,11 @@ class Regex:
     @property
     def nullable(self) -> bool:
         return bool(_load().orc_nullable(self._h))
+
+    @property
+    def max_len(self) -> int:
+        """Longest string of L(r) (an upper bound on match length); -1 = unbounded."""
+        return int(_load().orc_max_len(self._h))
 
     def run(self, data, use_cache: bool = True, max_states: int = 4096, dense: bool = True,
             positions: bool = False):
@@ -171,6 +178,17 @@ def run_set(patterns, data, threads: int | None = None, use_cache: bool = True, 
         raise OracleError(code, bad.value, 0, "pattern rejected by the oracle parser")
     return {"counts": counts[:n], "digests": digests[:n],
             "dense": dn[:n, :words] if dense else None, "threads": int(threads)}
+
+
+def positions_set(patterns, data, threads: int | None = None):
+    """Sorted match-end positions (u64 arrays) of every pattern over one
+    input, a thread pool over regexes (ctypes releases the GIL)."""
+    from concurrent.futures import ThreadPoolExecutor
+    buf = _as_u8(data)
+    regs = [Regex(p) for p in patterns]
+    with ThreadPoolExecutor(max_workers=threads or os.cpu_count() or 1) as ex:
+        res = list(ex.map(lambda r: r.run(buf, dense=False, positions=True)["positions"], regs))
+    return res
 
 
 def splitmix64(x: int) -> int:

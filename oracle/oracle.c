@@ -441,7 +441,41 @@ typedef struct orc_regex {
   uint64_t *after;    /* per state: closure({out}) for S_CHAR states (nw words each) */
   int match_state;
   int nullable;
+  int64_t max_len; /* longest string of L(r), -1 = unbounded (see ast_max_len) */
 } orc_regex;
+
+/* Longest string length of L(x) (an upper bound on the length of any match,
+ * used by the tests to window the oracle exactly: a match ending at i starts
+ * at >= i - max_len + 1); -1 = unbounded.  Straight from the grammar of
+ * Sec. 2: concatenation adds, alternation takes the maximum, a
+ * repetition multiplies its upper count, an unbounded repetition of a body
+ * that can consume a byte is unbounded. */
+static int64_t ast_max_len(const ast *x) {
+  int64_t a, b;
+  switch (x->kind) {
+    case A_EMPTY: return 0;
+    case A_SET: return 1;
+    case A_CAT:
+      a = ast_max_len(x->a);
+      b = ast_max_len(x->b);
+      return (a < 0 || b < 0) ? -1 : a + b;
+    case A_ALT:
+      a = ast_max_len(x->a);
+      b = ast_max_len(x->b);
+      return (a < 0 || b < 0) ? -1 : (a > b ? a : b);
+    case A_QUEST: return ast_max_len(x->a);
+    case A_STAR:
+    case A_PLUS:
+      a = ast_max_len(x->a);
+      return a == 0 ? 0 : -1;
+    case A_REP:
+      a = ast_max_len(x->a);
+      if (a == 0) return 0;
+      if (a < 0 || x->hi < 0) return -1;
+      return a * (int64_t)x->hi;
+  }
+  return -1;
+}
 
 static void closure_add(const orc_regex *r, int s, uint64_t *set, int *stack) {
   int sp = 0;
@@ -494,6 +528,7 @@ int orc_compile(const char *pat, size_t len, orc_regex **out, size_t *err_at, ch
         if (r->st[s].type == S_CHAR) closure_add(r, r->st[s].out, r->after + (size_t)s * r->nw, stack);
       free(stack);
       r->nullable = (int)((r->start[m >> 6] >> (m & 63)) & 1);
+      r->max_len = root ? ast_max_len(root) : 0;
       *out = r;
     }
   }
@@ -512,6 +547,7 @@ void orc_free(orc_regex *r) {
 
 int orc_num_states(const orc_regex *r) { return r->nst; }
 int orc_nullable(const orc_regex *r) { return r->nullable; }
+int64_t orc_max_len(const orc_regex *r) { return r->max_len; }
 
 /* One NFA step: nxt = closure(delta(src, c)); returns 1 iff MATCH in nxt. */
 static int nfa_step(const orc_regex *r, const uint64_t *src, int c, uint64_t *nxt) {

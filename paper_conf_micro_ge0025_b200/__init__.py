@@ -23,7 +23,7 @@ RX_F_NO_REBALANCE, RX_F_NO_GUARDS, RX_F_NO_CACHE, RX_F_REBALANCE, RX_F_NO_PREFIL
 
 EXPORTED = ["rx_compile", "rx_free", "rx_num_regex", "rx_num_groups", "rx_max_lookback", "rx_max_lookahead",
             "rx_boundary_bytes", "rx_program_source", "rx_program_info", "rx_match", "rx_match_chunk",
-            "rx_rematch_chunk", "rx_last_error", "rx_kernels_per_match"]
+            "rx_rematch_chunk", "rx_last_error", "rx_kernels_per_match", "rx_set_profiling", "rx_kernel_times"]
 
 
 class RxError(RuntimeError):
@@ -43,7 +43,8 @@ class _Error(ctypes.Structure):
 
 class _Output(ctypes.Structure):
     _fields_ = [("d_counts", ctypes.c_void_p), ("d_digests", ctypes.c_void_p), ("d_bitstreams", ctypes.c_void_p),
-                ("pitch_words", ctypes.c_uint64), ("d_status", ctypes.c_void_p), ("reserved", ctypes.c_uint32 * 4)]
+                ("pitch_words", ctypes.c_uint64), ("d_status", ctypes.c_void_p), ("d_matches", ctypes.c_void_p),
+                ("match_cap", ctypes.c_uint64), ("d_match_total", ctypes.c_void_p)]
 
 
 def lib_path() -> str:
@@ -79,6 +80,10 @@ def load_library():
         lib.rx_match_chunk.restype = ctypes.c_int
         lib.rx_rematch_chunk.argtypes = [vp, vp, u64, u64, u64, u64, vp, vp, vp, vp, ctypes.POINTER(_Output)]
         lib.rx_rematch_chunk.restype = ctypes.c_int
+        lib.rx_set_profiling.argtypes = [vp, ctypes.c_int]
+        lib.rx_set_profiling.restype = ctypes.c_int
+        lib.rx_kernel_times.argtypes = [vp, vp, vp, ctypes.c_int]
+        lib.rx_kernel_times.restype = ctypes.c_int
         lib.rx_last_error.argtypes = []
         lib.rx_last_error.restype = ctypes.c_char_p
         _lib = lib
@@ -166,13 +171,20 @@ class Program:
         return self._lib.rx_program_info(self._h).decode()
 
     # --- matching -----------------------------------------------------------
-    def alloc_outputs(self, length, device=None, dense=False, digests=True):
+    def alloc_outputs(self, length, device=None, dense=False, digests=True, match_cap=None):
+        """Output buffers of rx_output.  match_cap: None = no match list;
+        an int = a list of that many rx_match_t entries ({u32 regex, u32 pad,
+        u64 pos}, held as int64[cap, 2]) plus its u64 total; 0 = total only."""
         import torch
         device = device or torch.device("cuda", torch.cuda.current_device())
         n = self.n_regex
         out = {"counts": torch.zeros(max(n, 1), dtype=torch.int64, device=device)[:n],
                "digests": torch.zeros((max(n, 1), 2), dtype=torch.int64, device=device)[:n] if digests else None,
                "status": torch.zeros(1, dtype=torch.int32, device=device)}
+        if match_cap is not None:
+            out["matches"] = torch.zeros((max(int(match_cap), 1), 2), dtype=torch.int64, device=device)
+            out["match_cap"] = int(match_cap)
+            out["match_total"] = torch.zeros(1, dtype=torch.int64, device=device)
         if dense:
             pitch = max((int(length) + 31) // 32, 1)
             out["dense"] = torch.zeros((max(n, 1), pitch), dtype=torch.int32, device=device)[:n]
@@ -188,22 +200,40 @@ class Program:
         s.d_bitstreams = o["dense"].data_ptr() if o.get("dense") is not None else None
         s.pitch_words = int(o.get("pitch") or 0)
         s.d_status = o["status"].data_ptr() if o.get("status") is not None else None
+        if o.get("match_total") is not None:
+            s.d_match_total = o["match_total"].data_ptr()
+            s.d_matches = o["matches"].data_ptr() if o.get("match_cap") else None
+            s.match_cap = int(o.get("match_cap") or 0)
         return s
 
-    def match(self, data, out=None, dense=False, digests=True, stream=None):
+    @staticmethod
+    def match_list(out):
+        """(regex ids u32[m], positions u64[m]) of the listed matches, sorted
+        by (regex, position); raises if the list was truncated."""
+        import numpy as np
+        total = int(out["match_total"].cpu()[0])
+        if total > out["match_cap"]:
+            raise RxError(RX_EOVERFLOW, f"match list truncated: {total} matches > cap {out['match_cap']}")
+        a = out["matches"][:total].cpu().numpy().view(np.uint64)
+        reg, pos = (a[:, 0] & 0xFFFFFFFF).astype(np.uint32), a[:, 1].copy()
+        order = np.lexsort((pos, reg))
+        return reg[order], pos[order]
+
+    def match(self, data, out=None, dense=False, digests=True, match_cap=None, stream=None):
         """Match a CUDA uint8 tensor; returns dict(counts=int64[n] (u64 bits),
-        digests=int64[n,2], dense=int32[n, pitch] LSB-first, status)."""
+        digests=int64[n,2], dense=int32[n, pitch] LSB-first, status, and with
+        match_cap: matches / match_total -- see match_list())."""
         if out is None:
-            out = self.alloc_outputs(data.numel(), data.device, dense=dense, digests=digests)
+            out = self.alloc_outputs(data.numel(), data.device, dense=dense, digests=digests, match_cap=match_cap)
         s = self._out_struct(out)
         _check(self._lib.rx_match(self._h, _ptr(data), int(data.numel()), _stream_handle(stream), ctypes.byref(s)))
         return out
 
     def match_chunk(self, data, length, halo_left, halo_right, global_offset, state_in=None, state_out=None,
-                    out=None, accumulate=False, dense=False, digests=True, stream=None):
+                    out=None, accumulate=False, dense=False, digests=True, match_cap=None, stream=None):
         """`data` is a CUDA uint8 tensor holding [halo_left | chunk(length) | halo_right]."""
         if out is None:
-            out = self.alloc_outputs(length, data.device, dense=dense, digests=digests)
+            out = self.alloc_outputs(length, data.device, dense=dense, digests=digests, match_cap=match_cap)
         s = self._out_struct(out)
         base = data.data_ptr() + int(halo_left)
         _check(self._lib.rx_match_chunk(self._h, ctypes.c_void_p(base), int(length), int(halo_left), int(halo_right),
@@ -220,6 +250,16 @@ class Program:
                                           _ptr(state_true), _ptr(state_out), _stream_handle(stream),
                                           ctypes.byref(s)))
         return out
+
+    def set_profiling(self, on: bool = True):
+        _check(self._lib.rx_set_profiling(self._h, int(bool(on))))
+
+    def kernel_times(self, reset: bool = True):
+        """{kernel: (total ms, launches)} for prefilter / pass1 / fixup (rx_kernel_times)."""
+        ms = (ctypes.c_double * 3)()
+        n = (ctypes.c_uint64 * 3)()
+        _check(self._lib.rx_kernel_times(self._h, ms, n, int(bool(reset))))
+        return {k: (float(ms[i]), int(n[i])) for i, k in enumerate(("rx_prefilter", "rx_pass1", "rx_fixup"))}
 
     def new_state(self, device=None):
         import torch

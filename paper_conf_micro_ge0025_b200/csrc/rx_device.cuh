@@ -60,6 +60,10 @@ struct Ctx {
   bool want_digest, want_dense;
   const int *rid;  // group member -> global regex id
   u32 *status;
+  u64 *mlist;      // nullable: compacted match list, {regex, pos} pairs (rx_match_t)
+  u64 mcap;
+  u64 *mtotal;
+  u32 *fold;       // fix-up only: [NR][K] output words of the "old" run (match-list delta)
 };
 
 // ---------------------------------------------------------------------------
@@ -78,6 +82,61 @@ DEV u64 rx_warp_sum64(u64 v) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(RX_FULL, v, o);
   return v;
+}
+
+// Compacted match list (rx_output.d_matches): every set bit of the committed
+// words becomes one {regex, global position} entry; a warp reserves its slots
+// with one atomicAdd and each lane writes its own bits after an exclusive
+// prefix sum.  The fix-up's "old" run (sign = -1) records its words in c.fold
+// and the "new" run lists only the bits the old one lacked: match sets are
+// monotone in the incoming state (every operation on state streams is AND /
+// OR / Advance / add-with-carry of a marker into a class), so new covers old;
+// a violation is flagged in status bit 2 instead of being silently dropped.
+template <int K>
+DEV void rx_emit_list(const Ctx<K> &c, int r, const u32 (&m)[K]) {
+  u32 mm[K];
+  u32 cnt = 0;
+  bool lost = false;
+#pragma unroll
+  for (int i = 0; i < K; ++i) {
+    if (c.fold && c.sign == ~0ull) {
+      c.fold[r * K + i] = m[i];
+      mm[i] = 0u;
+    } else if (c.fold) {
+      lost = lost || (c.fold[r * K + i] & ~m[i]) != 0u;
+      mm[i] = m[i] & ~c.fold[r * K + i];
+    } else {
+      mm[i] = m[i];
+    }
+    cnt += __popc(mm[i]);
+  }
+  if (lost) atomicOr(c.status, 4u);
+  u32 incl = cnt;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const u32 t = __shfl_up_sync(RX_FULL, incl, o);
+    if (c.lane >= (u32)o) incl += t;
+  }
+  const u32 tot = __shfl_sync(RX_FULL, incl, 31);
+  if (tot == 0u) return;
+  u64 base = 0;
+  if (c.lane == 0) base = atomicAdd(c.mtotal, (u64)tot);
+  base = __shfl_sync(RX_FULL, base, 0) + (incl - cnt);
+  const u64 reg = (u64)(u32)c.rid[r];
+#pragma unroll
+  for (int i = 0; i < K; ++i) {
+    u32 b = mm[i];
+    const i64 wpos = c.gofs + (c.word0 + (i64)(c.lane * K + i)) * 32;
+    while (b) {
+      const int t = __ffs(b) - 1;
+      b &= b - 1u;
+      if (base < c.mcap) {
+        c.mlist[2 * base] = reg;
+        c.mlist[2 * base + 1] = (u64)(wpos + t);
+      }
+      ++base;
+    }
+  }
 }
 
 template <int K>
@@ -122,6 +181,7 @@ __device__ __noinline__ void rx_emit(const Ctx<K> c, int r, const V<K> v) {
     c.acc[3 * r + 1] += c.sign * d1;
     c.acc[3 * r + 2] += c.sign * d2;
   }
+  if (c.mtotal) rx_emit_list<K>(c, r, m);
 }
 
 // ---------------------------------------------------------------------------
@@ -196,6 +256,9 @@ struct RxParams {
   int pf_aligned;           // in + avail_lo is 16-byte aligned
   u64 *stats;               // nullable: debug counters (RX_STATS=1), see rx_run_segment_pf
   int dbg;                  // timing experiments only (RX_DBG): 1 = skip every window, 2 = no body
+  u64 *matches;             // nullable: rx_match_t[match_cap] as u64 pairs {regex, pos}
+  u64 match_cap;
+  u64 *match_total;         // u64: matches found (may exceed match_cap)
 };
 
 template <int K> DEV void rx_load_window(const RxParams &p, Ctx<K> &c, u32 (&pl)[8][K], i64 fword) {
@@ -349,6 +412,10 @@ template <class G> DEV void rx_ctx_init(const RxParams &p, Ctx<G::K> &c, u64 *ac
   c.want_dense = p.dense != nullptr;
   c.rid = G::rid();
   c.status = p.status;
+  c.mlist = p.matches;
+  c.mcap = p.match_cap;
+  c.mtotal = p.match_total;
+  c.fold = nullptr;
   for (int r = (int)c.lane; r < 3 * G::NR; r += 32) acc[r] = 0ull;
   __syncwarp();
 }
@@ -559,6 +626,8 @@ DEV void rx_fixup_group(const RxParams &p, u64 *acc, u32 *sst) {
   u32 pl[8][K];
   u32 xr[K][8];
   u32 *tru = sst, *old = sst + M, *t1 = sst + 2 * M, *t2 = sst + 3 * M;
+  u32 fold[G::NR * K];
+  c.fold = p.match_total ? fold : nullptr;
   for (int s = (int)c.lane; s < NS; s += 32) {
     tru[s] = p.st_in ? p.st_in[G::SBASE + s] : 0u;
     old[s] = (p.mode == 2 && p.st_assumed) ? p.st_assumed[G::SBASE + s] : 0u;
@@ -585,6 +654,8 @@ DEV void rx_fixup_group(const RxParams &p, u64 *acc, u32 *sst) {
       // old run: subtract
       c.sign = ~0ull;
       c.want_dense = false;
+      if (c.fold)
+        for (int j = 0; j < G::NR * K; ++j) fold[j] = 0u;
       rx_state_zero(t1, NS, c.lane);
       G::body(c, pl, old, t1, ~0u);
       // new run: add, rewrite dense words

@@ -131,8 +131,12 @@ void write_file_atomic(const std::string &path, const std::string &data) {
 bool nvrtc_compile(const std::string &src, int max_regs, bool use_cache, std::string &cubin, std::string &log) {
   int maj = 0, mnr = 0;
   nvrtcVersion(&maj, &mnr);
-  std::vector<std::string> opts = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo", "-default-device",
-                                   "-rdc=true", "--maxrregcount=" + std::to_string(max_regs), "-DNDEBUG"};
+  // -lineinfo only on request (RX_LINEINFO=1, for ncu source pages): in -rdc
+  // mode it embeds the PTX text and makes each group unit ~4x larger
+  std::vector<std::string> opts = {"--gpu-architecture=sm_100a", "-std=c++17", "-default-device", "-rdc=true",
+                                   "--maxrregcount=" + std::to_string(max_regs), "-DNDEBUG"};
+  const char *li = getenv("RX_LINEINFO");
+  if (li && *li == '1') opts.push_back("-lineinfo");
   std::string key_src = src;
   for (auto &o : opts) key_src += "\n//" + o;
   key_src += "\n//nvrtc " + std::to_string(maj) + "." + std::to_string(mnr);
@@ -199,6 +203,16 @@ struct rx_program {
   std::string all_source;
   std::string info;
   std::mutex mu;
+  // per-kernel timing (rx_set_profiling): CUDA events recorded on the launch
+  // stream around every launch; kinds 0 = prefilter, 1 = pass 1, 2 = fix-up
+  bool prof = false;
+  struct Ev {
+    int kind;
+    cudaEvent_t a, b;
+  };
+  std::vector<Ev> prof_ev;
+  double prof_ms[3] = {0, 0, 0};
+  uint64_t prof_n[3] = {0, 0, 0};
 };
 
 extern "C" {
@@ -218,6 +232,37 @@ uint32_t rx_kernels_per_match(const rx_program *p) {
   return n;
 }
 const char *rx_program_info(const rx_program *p) { return p ? p->info.c_str() : ""; }
+
+rx_status rx_set_profiling(rx_program *p, int on) {
+  if (!p) return fail(RX_EINVAL, "null program");
+  std::lock_guard<std::mutex> lk(p->mu);
+  p->prof = on != 0;
+  return RX_OK;
+}
+
+rx_status rx_kernel_times(rx_program *p, double *ms, uint64_t *launches, int reset) {
+  if (!p) return fail(RX_EINVAL, "null program");
+  std::lock_guard<std::mutex> lk(p->mu);
+  for (auto &e : p->prof_ev) {
+    float t = 0.f;
+    if (cudaEventSynchronize(e.b) != cudaSuccess || cudaEventElapsedTime(&t, e.a, e.b) != cudaSuccess)
+      return fail(RX_ECUDA, "event timing failed");
+    p->prof_ms[e.kind] += t;
+    p->prof_n[e.kind] += 1;
+    cudaEventDestroy(e.a);
+    cudaEventDestroy(e.b);
+  }
+  p->prof_ev.clear();
+  for (int k = 0; k < 3; ++k) {
+    if (ms) ms[k] = p->prof_ms[k];
+    if (launches) launches[k] = p->prof_n[k];
+    if (reset) {
+      p->prof_ms[k] = 0;
+      p->prof_n[k] = 0;
+    }
+  }
+  return RX_OK;
+}
 
 void rx_free(rx_program *p) {
   if (!p) return;
@@ -445,6 +490,9 @@ struct RxParamsHost {  // must mirror RxParams in rx_device.cuh
   int pf_aligned;
   unsigned long long *stats;
   int dbg;
+  unsigned long long *matches;
+  unsigned long long match_cap;
+  unsigned long long *match_total;
 };
 
 rx_status ensure_loaded(rx_program *p, int &device) {
@@ -495,10 +543,16 @@ rx_status ensure_loaded(rx_program *p, int &device) {
 constexpr int kPass1Warps = 16;  // one CTA = one SM's worth of warps, one group (lockstep)
 constexpr int kFixupWarps = 4;
 
-rx_status launch(RxModule &m, CUfunction f, long long blocks, int warps_per_block, const RxParamsHost &prm,
-                 cudaStream_t s) {
+rx_status launch(rx_program *p, RxModule &m, CUfunction f, long long blocks, int warps_per_block,
+                 const RxParamsHost &prm, cudaStream_t s) {
   Drv &d = drv();
   if (blocks <= 0) return RX_OK;
+  rx_program::Ev ev{f == m.prefilter ? 0 : (f == m.pass1 ? 1 : 2), nullptr, nullptr};
+  if (p->prof) {
+    cudaEventCreate(&ev.a);
+    cudaEventCreate(&ev.b);
+    cudaEventRecord(ev.a, s);
+  }
   if (blocks > 0x7fffffffLL) return fail(RX_EINVAL, "grid too large");
   // must match the layout emitted in rx_codegen.cpp (accumulators | state |
   // TMA window staging | mbarriers); the fix-up kernel uses the first two
@@ -513,6 +567,11 @@ rx_status launch(RxModule &m, CUfunction f, long long blocks, int warps_per_bloc
   void *args[] = {&local};
   CUresult r =
       d.LaunchKernel(f, (unsigned)blocks, 1, 1, 32 * warps_per_block, 1, 1, smem, (CUstream)s, args, nullptr);
+  if (p->prof) {
+    cudaEventRecord(ev.b, s);
+    std::lock_guard<std::mutex> lk(p->mu);
+    p->prof_ev.push_back(ev);
+  }
   if (r != CUDA_SUCCESS) return fail(RX_ECUDA, "cuLaunchKernel failed: " + std::to_string((int)r));
   return RX_OK;
 }
@@ -539,6 +598,8 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
         cudaMemsetAsync(out->d_bitstreams, 0, 4ull * n * out->pitch_words, stream) != cudaSuccess)
       return fail(RX_ECUDA, "memset");
     if (out->d_status && cudaMemsetAsync(out->d_status, 0, 4, stream) != cudaSuccess) return fail(RX_ECUDA, "memset");
+    if (out->d_match_total && cudaMemsetAsync(out->d_match_total, 0, 8, stream) != cudaSuccess)
+      return fail(RX_ECUDA, "memset");
   }
   RxParamsHost prm;
   memset(&prm, 0, sizeof prm);
@@ -561,6 +622,10 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
   prm.st_assumed = (const unsigned int *)st_assumed;
   prm.aligned = (((uintptr_t)d_input) & 15) == 0 ? 1 : 0;
   prm.accumulate = accumulate;
+  if (out->d_matches && !out->d_match_total) return fail(RX_EINVAL, "d_matches needs d_match_total");
+  prm.matches = (unsigned long long *)out->d_matches;
+  prm.match_cap = out->d_matches ? out->match_cap : 0;
+  prm.match_total = (unsigned long long *)out->d_match_total;
   {
     const char *e = getenv("RX_LOCKSTEP");  // experiment knob: 0 = no per-window CTA barrier
     prm.lockstep = (e && *e == '0') ? 0 : 1;
@@ -582,7 +647,7 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
     for (auto &m : p->mods) {
       if (!m.any_state) continue;
       prm.seg_state = nullptr;
-      s = launch(m, m.fixup, div_up(m.g_end - m.g_begin, kFixupWarps), kFixupWarps, prm, stream);
+      s = launch(p, m, m.fixup, div_up(m.g_end - m.g_begin, kFixupWarps), kFixupWarps, prm, stream);
       if (s != RX_OK) return s;
     }
     if (status_scratch) cudaFreeAsync(status_scratch, stream);
@@ -633,7 +698,7 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
         const char *e = getenv("RX_PF_LOCKSTEP");  // experiment knob
         prm.lockstep = (e && *e == '1') ? 1 : 0;
       }
-      s = launch(m, m.prefilter, std::min<long long>(ntiles, 148LL * 4), 16, prm, stream);
+      s = launch(p, m, m.prefilter, std::min<long long>(ntiles, 148LL * 4), 16, prm, stream);
       if (s != RX_OK) return s;
     }
     unsigned long long *stats = nullptr;
@@ -644,7 +709,7 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
       const char *de = getenv("RX_DBG");  // timing experiments only: results are wrong when set
       prm.dbg = (de && *de) ? atoi(de) : 0;
     }
-    s = launch(m, m.pass1, cpg * mg, kPass1Warps, prm, stream);
+    s = launch(p, m, m.pass1, cpg * mg, kPass1Warps, prm, stream);
     prm.stats = nullptr;
     if (stats) {
       unsigned long long h[8];
@@ -659,7 +724,7 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
     if (s != RX_OK) return s;
     if (m.any_state) {
       prm.mode = 1;
-      s = launch(m, m.fixup, div_up(mg, kFixupWarps), kFixupWarps, prm, stream);
+      s = launch(p, m, m.fixup, div_up(mg, kFixupWarps), kFixupWarps, prm, stream);
       if (s != RX_OK) return s;
       cudaFreeAsync(seg_state, stream);
     }

@@ -154,3 +154,28 @@ def test_chunked_speculative_then_rematch():
     dig = sum(o["digests"].cpu().numpy().view(np.uint64) for o in outs)
     assert np.array_equal(tot, whole["counts"])
     assert np.array_equal(dig, whole["digests"])
+
+
+def test_match_list_equals_oracle_positions():
+    # several segments per group (so the carry fix-up runs and lists only
+    # the matches the speculative pass lacked), the 20 KB a(bc)*d chain
+    # crossing segment boundaries, .* state crossing many windows
+    pats = gen.tiny_patterns() + [rb"abcd.*xyz", rb"q[^z]*z", rb"(ab|cd)+e"]
+    data = gen.tiny_input() * 8
+    prog = rx.Program(pats)
+    d = torch.frombuffer(bytearray(data), dtype=torch.uint8).cuda()
+    out = prog.match(d, match_cap=1 << 20)
+    torch.cuda.synchronize()
+    assert int(out["status"].cpu()[0]) == 0
+    reg, pos = prog.match_list(out)
+    counts = out["counts"].cpu().numpy().view(np.uint64)
+    assert reg.size == int(counts.sum()) > 0
+    for r, p in enumerate(pats):
+        want = oracle.Regex(p).run(data, dense=False, positions=True)["positions"]
+        assert np.array_equal(pos[reg == r], want), p
+    # truncated list: the total is still exact, the call reports it
+    out2 = prog.match(d, match_cap=10)
+    torch.cuda.synchronize()
+    assert int(out2["match_total"].cpu()[0]) == reg.size
+    with pytest.raises(rx.RxError):
+        prog.match_list(out2)

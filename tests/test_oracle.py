@@ -243,3 +243,25 @@ def test_tiny_long_chain_is_found():
                                       (b"(?=a)", 2), (b"\\bx", 2), (b"a{2000}", 3), (b"\\q", 1)])
 def test_rejected_constructs(pat, code):
     assert oracle.check(pat)[0] == code
+
+
+@pytest.mark.parametrize("pat,want", [(b"abc", 3), (b"a{2,5}", 5), (b"(ab|c)+", -1), (b"a?|bcd", 3), (b"a*|bcd", -1),
+                                      (b"x(ab){3}y?", 8), (b"[0-9]+x", -1), (b"(a?){4}", 4), (b"()*", 0),
+                                      (b"a.{0,32}b", 34), (b"(foo|ba[rz])", 3)])
+def test_max_len_closed_forms(pat, want):
+    assert oracle.Regex(pat).max_len == want
+
+
+def test_max_len_bounds_every_brute_force_match():
+    # the longest match found by brute force (all starts, all ends) never
+    # exceeds max_len, and reaches it on a text made of the longest member
+    rng = np.random.default_rng(777)
+    for _ in range(150):
+        p = gen.fuzz_pattern(rng)
+        ml = oracle.Regex(p).max_len
+        t = gen.fuzz_text(rng, int(rng.integers(1, 12 if _nested_repeat(p) else 30)))
+        rx = re.compile(p)
+        longest = max([i + 1 - s for i in range(len(t)) for s in range(i + 1) if rx.fullmatch(t, s, i + 1)],
+                      default=0)
+        if ml >= 0:
+            assert longest <= ml, (p, t, longest, ml)
