@@ -43,6 +43,8 @@ struct RegexEmitter {
   std::vector<std::map<TabKey, std::string>> &cc_scope;
   std::vector<std::map<std::vector<uint64_t>, std::string>> &set_scope;
   int tmp = 0;
+  std::string lit_pool;          // name of the group's literal byte table
+  std::vector<int> lit_off;      // offset of ir.lits[i] in it
 
   RegexEmitter(std::ostringstream &o, const RegexIR &r, int k, int rl, int sb,
                std::vector<std::map<TabKey, std::string>> &ccs,
@@ -277,6 +279,16 @@ struct RegexEmitter {
         }
         break;
       case Op::Look: look(in, nv(id), A, n.k); break;
+      case Op::Lit: {
+        // literal run confirmed byte by byte at the (sparse) marker bits
+        std::string t = fresh();
+        os << I << "V<" << K << "> " << t << "i;\n";
+        for (int i = 0; i < K; ++i) os << I << t << "i.w[" << i << "] = " << W(A, i) << ";\n";
+        os << I << "const V<" << K << "> " << t << "o = rx_lit<" << K << ">(c, " << t << "i, " << lit_pool << " + "
+           << lit_off[n.cc] << ", " << n.k << ");\n";
+        decl(in, nv(id), [&](int i) { return t + "o.w[" + std::to_string(i) + "]"; });
+        break;
+      }
       case Op::MStar:
         if (n.loop >= 0)
           mstar(in, nv(id), A, B, n.aw, "(" + first + " ? " + st(n.slot) + " : 0u)", nst(n.slot), true);
@@ -388,7 +400,8 @@ struct RegexEmitter {
       case Op::Ones: case Op::CC: case Op::Fr: return false;
       case Op::And: return zero_when_unfired(n.a) || zero_when_unfired(n.b);
       case Op::Or: case Op::Xor: return zero_when_unfired(n.a) && zero_when_unfired(n.b);
-      case Op::AndNot: case Op::Adv: case Op::Look: case Op::MStar: case Op::Loop: return zero_when_unfired(n.a);
+      case Op::AndNot: case Op::Adv: case Op::Look: case Op::MStar: case Op::Loop: case Op::Lit:
+        return zero_when_unfired(n.a);
     }
     return false;
   }
@@ -471,6 +484,12 @@ static void layout(const CompiledSet &cs, int &nsmax, int &nrmax) {
     nrmax = std::max(nrmax, (int)g.regexes.size());
   }
 }
+// per-warp shared bytes of the literal-run scratch (frame bytes + output words)
+int lit_scratch_bytes(const CompiledSet &cs) {
+  int kmax = 1;
+  for (auto &g : cs.groups) kmax = std::max(kmax, g.K);
+  return 1152 * kmax;
+}
 
 // One relocatable compilation unit per group (NVRTC -rdc): the group's
 // traits, its program body, and the two non-inlined entry functions
@@ -487,6 +506,18 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
   for (int h = 0; h < gi; ++h) sbase += cs.groups[h].nslots;
   {
     Group &g = cs.groups[gi];
+    // the group's literal runs (Op::Lit), one byte table
+    std::vector<std::vector<int>> lit_off(g.clusters.size());
+    std::string pool;
+    for (size_t ci = 0; ci < g.clusters.size(); ++ci)
+      for (auto &l : g.clusters[ci].ir.lits) {
+        lit_off[ci].push_back((int)pool.size());
+        pool += l;
+      }
+    os << "__device__ const unsigned char rx_litb_" << gi << "[" << std::max<size_t>(pool.size(), 1) << "] = {";
+    for (size_t i = 0; i < pool.size(); ++i) os << (i ? "," : "") << (unsigned)(unsigned char)pool[i];
+    if (pool.empty()) os << "0";
+    os << "};\n";
     os << "__device__ const int rx_rid_" << gi << "[" << g.regexes.size() << "] = {";
     for (size_t i = 0; i < g.regexes.size(); ++i) os << (i ? "," : "") << g.regexes[i];
     os << "};\n";
@@ -497,10 +528,13 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
     os << "  static DEV const int *rid() { return rx_rid_" << gi << "; }\n";
     os << "  static constexpr unsigned ALWAYS = " << g.always << "u;\n";
     os << "  static constexpr bool PF = " << (cs.use_pf ? "true" : "false") << ";\n";
+    os << "  static constexpr bool LIT = " << (pool.empty() ? "false" : "true") << ";\n";
     // rmask: members whose prefilter factor occurs in the window frame
     // (rx_prefilter); members without a factor (ALWAYS) and members carrying
     // state into the window run regardless
-    os << "  static DEV void body(Ctx<" << g.K << "> &c, const u32 (&pl)[8][" << g.K
+    // one out-of-line copy shared by pass 1 and both fix-up runs (code size,
+    // NVRTC time; the call costs nothing next to the body)
+    os << "  static __device__ __noinline__ void body(Ctx<" << g.K << "> &c, const u32 (&pl)[8][" << g.K
        << "], const u32 *st, u32 *nst, const u32 rmask) {\n";
     os << "    (void)st; (void)nst; (void)rmask;\n";
     os << "    const u32 lane = c.lane; const int cw = (int)c.cw; (void)cw;\n";
@@ -515,6 +549,8 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
       const Cluster &cl = g.clusters[ci];
       RegexEmitter em(os, cl.ir, g.K, (int)ci, cl.slot_base, ccs, sets);
       em.out_member = cl.members;
+      em.lit_pool = "rx_litb_" + std::to_string(gi);
+      em.lit_off = lit_off[ci];
       std::string run;
       if (cl.always) {
         run = "true";
@@ -540,24 +576,31 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
       os << "    }\n";
     }
     os << "  }\n};\n";
+    const int LB = lit_scratch_bytes(cs);
     os << "extern \"C\" __device__ __noinline__ void rx_seg_" << gi
        << "(const RxParams &p, int seg) {\n"
-       // shared memory: [wpb][3*NRMAX] u64 accumulators | [wpb][4*NSMAX] u32 state |
-       // [wpb][2][2048] window staging (TMA) | [wpb][2] u64 mbarriers
+       // shared memory (rx_runtime.cpp launch() mirrors it): [wpb][3*NRMAX] u64
+       // accumulators | [wpb][4*NSMAX] u32 state | [wpb][LB] literal-run
+       // scratch | [wpb][4096] window staging (TMA) | [wpb][2] u64 mbarriers
        << "  extern __shared__ __align__(16) u64 rx_smem[];\n"
        << "  const int warp = threadIdx.x >> 5, wpb = blockDim.x >> 5;\n"
        << "  u64 *acc = rx_smem + warp * (3 * " << nrmax << ");\n"
        << "  u32 *st0 = reinterpret_cast<u32 *>(rx_smem + wpb * (3 * " << nrmax << "));\n"
-       << "  unsigned char *tb0 = reinterpret_cast<unsigned char *>(st0 + ((wpb * (4 * " << nsmax
+       << "  unsigned char *lb0 = reinterpret_cast<unsigned char *>(st0 + ((wpb * (4 * " << nsmax
        << ") + 3) & ~3));\n"
+       << "  unsigned char *tb0 = lb0 + wpb * " << LB << ";\n"
        << "  u64 *bars = reinterpret_cast<u64 *>(tb0 + wpb * 4096) + 2 * warp;\n"
-       << "  rx_run_segment<RxG" << gi << ">(p, seg, acc, st0 + warp * (4 * " << nsmax << "), tb0 + warp * 4096, bars);\n}\n";
+       << "  rx_run_segment<RxG" << gi << ">(p, seg, acc, st0 + warp * (4 * " << nsmax
+       << "), tb0 + warp * 4096, bars, lb0 + warp * " << LB << ");\n}\n";
     if (g.nslots > 0)
-      os << "extern \"C\" __device__ __noinline__ void rx_fix_" << gi << "(const RxParams &p) {\n"
-         << "  extern __shared__ u64 rx_smem[];\n"
+      os << "extern \"C\" __device__ __noinline__ void rx_fix_" << gi << "(const RxParams &p, int seg) {\n"
+         << "  extern __shared__ __align__(16) u64 rx_smem[];\n"
          << "  const int warp = threadIdx.x >> 5, wpb = blockDim.x >> 5;\n"
-         << "  rx_fixup_group<RxG" << gi << ">(p, rx_smem + warp * (3 * " << nrmax << "),\n"
-         << "      reinterpret_cast<u32 *>(rx_smem + wpb * (3 * " << nrmax << ")) + warp * (4 * " << nsmax << "));\n}\n";
+         << "  u32 *st0 = reinterpret_cast<u32 *>(rx_smem + wpb * (3 * " << nrmax << "));\n"
+         << "  unsigned char *lb0 = reinterpret_cast<unsigned char *>(st0 + ((wpb * (4 * " << nsmax
+         << ") + 3) & ~3));\n"
+         << "  rx_fixup_group<RxG" << gi << ">(p, rx_smem + warp * (3 * " << nrmax << "), st0 + warp * (4 * " << nsmax
+         << "), lb0 + warp * " << LB << ", seg);\n}\n";
   }
   return os.str();
 }
@@ -574,7 +617,7 @@ std::string emit_kernel_unit(CompiledSet &cs) {
   os << "#define RX_NG " << G << "\n#define RX_NSMAX " << nsmax << "\n#define RX_NRMAX " << nrmax << "\n";
   for (int gi = 0; gi < G; ++gi) {
     os << "extern \"C\" __device__ void rx_seg_" << gi << "(const RxParams &p, int seg);\n";
-    if (cs.groups[gi].nslots > 0) os << "extern \"C\" __device__ void rx_fix_" << gi << "(const RxParams &p);\n";
+    if (cs.groups[gi].nslots > 0) os << "extern \"C\" __device__ void rx_fix_" << gi << "(const RxParams &p, int seg);\n";
   }
   int g_begin = 0;
   // pass 1: one CTA of 16 warps (the whole SM's register file) runs one
@@ -596,11 +639,14 @@ std::string emit_kernel_unit(CompiledSet &cs) {
   os << "\nextern \"C\" __global__ void __launch_bounds__(128) rx_fixup(const RxParams p) {\n"
         "  const int warp = threadIdx.x >> 5;\n"
         "  const int wpb = blockDim.x >> 5;\n"
-        "  const long long g = (long long)blockIdx.x * wpb + warp;\n"
+        "  const long long gw = (long long)blockIdx.x * wpb + warp;\n"
+        "  // phase 1: warp -> (group, segment); otherwise warp -> group\n"
+        "  const long long g = p.fix_phase == 1 ? gw / p.nseg_max : gw;\n"
+        "  const int seg = p.fix_phase == 1 ? (int)(gw % p.nseg_max) : 0;\n"
         "  if (g >= RX_NG) return;\n"
         "  switch ((int)g) {\n";
   for (int gi = 0; gi < G; ++gi)
-    if (cs.groups[g_begin + gi].nslots > 0) os << "    case " << gi << ": rx_fix_" << gi << "(p); break;\n";
+    if (cs.groups[g_begin + gi].nslots > 0) os << "    case " << gi << ": rx_fix_" << gi << "(p, seg); break;\n";
   os << "    default: break;\n  }\n}\n";
   return os.str();
 }

@@ -64,6 +64,8 @@ struct Ctx {
   u64 mcap;
   u64 *mtotal;
   u32 *fold;       // fix-up only: [NR][K] output words of the "old" run (match-list delta)
+  unsigned char *wb;  // nullable (groups without literal runs): the frame's bytes, frame position f at wb[f]
+  u32 *ob;            // literal-run output scratch, 32*K words (per warp)
 };
 
 // ---------------------------------------------------------------------------
@@ -185,6 +187,55 @@ __device__ __noinline__ void rx_emit(const Ctx<K> c, int r, const V<K> v) {
 }
 
 // ---------------------------------------------------------------------------
+// literal run (IR Op::Lit): out[p] = v[p-n] &
+// (bytes p-n+1..p == lit[0..n)), the exact result of the chain
+// v_j = Adv(v_{j-1}, 1) & CC(lit[j-1]) (Fig. 2b/2c), evaluated at
+// the marker bits only: each lane confirms its own bits against the frame's
+// bytes in shared memory and ORs the hits into a per-warp word buffer.
+// Output bits beyond the frame fall off, as the advances would shift them
+// out; the literal holds no 0x00 byte, so positions outside the stream
+// (read as 0) never confirm.
+// ---------------------------------------------------------------------------
+template <int K>
+__device__ __noinline__ V<K> rx_lit(const Ctx<K> &c, const V<K> v, const unsigned char *lit, int n) {
+  V<K> r;
+  u32 any = 0u;
+#pragma unroll
+  for (int i = 0; i < K; ++i) any |= v.w[i];
+  if (!__any_sync(RX_FULL, any != 0u)) {
+#pragma unroll
+    for (int i = 0; i < K; ++i) r.w[i] = 0u;
+    return r;
+  }
+  u32 *ob = c.ob;
+#pragma unroll
+  for (int i = 0; i < K; ++i) ob[c.lane * K + i] = 0u;
+  __syncwarp();
+  const unsigned char *wb = c.wb;
+  const int F = 1024 * K;
+  const unsigned char l0 = lit[0];
+#pragma unroll
+  for (int i = 0; i < K; ++i) {
+    u32 b = v.w[i];
+    while (b) {
+      const int t = __ffs(b) - 1;
+      b &= b - 1u;
+      const int q = (int)((c.lane * K + i) * 32u) + t;
+      const int e = q + n;
+      if (e >= F || wb[q + 1] != l0) continue;
+      int j = 1;
+      while (j < n && wb[q + 1 + j] == lit[j]) ++j;
+      if (j == n) atomicOr(&ob[e >> 5], 1u << (e & 31));
+    }
+  }
+  __syncwarp();
+#pragma unroll
+  for (int i = 0; i < K; ++i) r.w[i] = ob[c.lane * K + i];
+  __syncwarp();
+  return r;
+}
+
+// ---------------------------------------------------------------------------
 // prologue: load + fused transposition
 // ---------------------------------------------------------------------------
 // 32 bytes x[0..7] (little-endian words) -> 8 basis words: plane[k] bit j =
@@ -250,7 +301,8 @@ struct RxParams {
   u32 pf_hbits;             // log2 hash slots
   int pf_tab_smem;          // the whole blob is staged in shared memory
   u32 *pf_gbits;            // [NG][ntiles]: bit b of word t = factor of the group in block 32t+b
-  unsigned short *pf_blist; // [nblk][16]: hit count, then up to 15 factor ids (written for blocks with hits)
+  u32 *pf_mmask;            // [NG][32*ntiles]: members of the group whose factor occurs in the block
+                            // (written only where non-zero: read only where the pf_gbits bit is set)
   i64 pf_ntiles;
   int pf_on;
   int pf_aligned;           // in + avail_lo is 16-byte aligned
@@ -259,6 +311,9 @@ struct RxParams {
   u64 *matches;             // nullable: rx_match_t[match_cap] as u64 pairs {regex, pos}
   u64 match_cap;
   u64 *match_total;         // u64: matches found (may exceed match_cap)
+  int fix_phase;            // mode 1: 0 = serial fix-up, 1 = parallel per segment, 2 = serial remainder
+  u32 *seg_fix;             // [nseg_max][G][NSMAX]: phase-1 end state of a segment that did not converge
+  u32 *seg_nc;              // [nseg_max][G]: that segment did not converge in phase 1
 };
 
 template <int K> DEV void rx_load_window(const RxParams &p, Ctx<K> &c, u32 (&pl)[8][K], i64 fword) {
@@ -353,6 +408,11 @@ DEV void rx_unpack(const RxParams &p, const RxRange &ir, Ctx<K> &c, const u32 (&
   const bool interior = fword >= ir.lo && fword + 32 * K <= ir.hi;
 #pragma unroll
   for (int i = 0; i < K; ++i) {
+    if (c.wb) {  // raw frame bytes for literal runs (rx_lit)
+      uint4 *d = reinterpret_cast<uint4 *>(c.wb + (c.lane * K + i) * 32u);
+      d[0] = make_uint4(x[i][0], x[i][1], x[i][2], x[i][3]);
+      d[1] = make_uint4(x[i][4], x[i][5], x[i][6], x[i][7]);
+    }
     u32 t[8];
     rx_transpose32(x[i], t);
 #pragma unroll
@@ -401,7 +461,7 @@ template <class G> DEV void rx_flush(const RxParams &p, const Ctx<G::K> &c) {
   }
 }
 
-template <class G> DEV void rx_ctx_init(const RxParams &p, Ctx<G::K> &c, u64 *acc) {
+template <class G> DEV void rx_ctx_init(const RxParams &p, Ctx<G::K> &c, u64 *acc, unsigned char *lb) {
   c.lane = rx_lane();
   c.acc = acc;
   c.dense = p.dense;
@@ -416,6 +476,8 @@ template <class G> DEV void rx_ctx_init(const RxParams &p, Ctx<G::K> &c, u64 *ac
   c.mcap = p.match_cap;
   c.mtotal = p.match_total;
   c.fold = nullptr;
+  c.wb = G::LIT ? lb : nullptr;
+  c.ob = G::LIT ? reinterpret_cast<u32 *>(lb + 1024 * G::K) : nullptr;
   for (int r = (int)c.lane; r < 3 * G::NR; r += 32) acc[r] = 0ull;
   __syncwarp();
 }
@@ -448,6 +510,9 @@ DEV void rx_mbar_init(u64 *bar, u32 count) {
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
 }
 DEV void rx_bulk_load(void *dst, const void *src, u32 bytes, u64 *bar) {
+  // the warp's generic-proxy reads of dst (ordered by the caller's
+  // __syncwarp) must precede the async-proxy write
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(rx_smem_addr(bar)), "r"(bytes)
                : "memory");
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
@@ -469,17 +534,20 @@ DEV void rx_mbar_wait(u64 *bar, u32 phase) {
 // Runs one group (traits G) over one segment (pass 1).  Windows of groups
 // with K <= 2 are staged through shared memory by TMA bulk copies issued
 // one window ahead; wider groups prefetch into registers.
-template <class G> DEV void rx_run_segment_pf(const RxParams &p, int seg, u64 *acc, u32 *sst);
+template <class G> DEV void rx_run_segment_pf(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *lb);
+template <class G>
+DEV void rx_run_segment_pf_staged(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *tbuf, u64 *bar,
+                                  unsigned char *lb);
 
 template <class G>
-DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *tbuf, u64 *bars) {
+DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *tbuf, u64 *bars,
+                        unsigned char *lb) {
   constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS;
   constexpr u32 WB = 1024u * K;  // window bytes
   if constexpr (G::PF) {
-    (void)tbuf;
-    (void)bars;
     (void)WB;
-    rx_run_segment_pf<G>(p, seg, acc, sst);
+    if (K <= 4 && !p.lockstep && !p.dbg) rx_run_segment_pf_staged<G>(p, seg, acc, sst, tbuf, bars, lb);
+    else rx_run_segment_pf<G>(p, seg, acc, sst, lb);
     return;
   }
   if constexpr (K <= 2) {
@@ -489,7 +557,7 @@ DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned
     const bool live = w_begin < nwin || seg == 0;
     const i64 w_end = !live ? w_begin : (w_begin + p.sw < nwin ? w_begin + p.sw : nwin);
     Ctx<K> c;
-    rx_ctx_init<G>(p, c, acc);
+    rx_ctx_init<G>(p, c, acc, lb);
     u32 pl[8][K];
     u32 xr[K][8];
     u32 *st = sst, *nst = sst + G::NSMAX;
@@ -571,7 +639,7 @@ DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned
   const bool live = w_begin < nwin || seg == 0;
   const i64 w_end = !live ? w_begin : (w_begin + p.sw < nwin ? w_begin + p.sw : nwin);
   Ctx<K> c;
-  rx_ctx_init<G>(p, c, acc);
+  rx_ctx_init<G>(p, c, acc, lb);
   u32 pl[8][K];
   u32 xr[K][8];
   u32 *st = sst, *nst = sst + G::NSMAX;
@@ -615,34 +683,27 @@ DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned
 // the true state; wherever it differs from the state pass 1 used, re-run the
 // window with both states and apply (new - old) until they agree.
 template <class G>
-DEV void rx_fixup_group(const RxParams &p, u64 *acc, u32 *sst) {
+DEV void rx_fixup_group(const RxParams &p, u64 *acc, u32 *sst, unsigned char *lb, int fseg) {
   constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS, M = G::NSMAX;
   if (NS == 0) return;
   const i64 len_words = rx_div_up(p.len, 32);
   const i64 nwin = rx_div_up(len_words, Bw);
   const i64 nseg = rx_div_up(nwin, p.sw);
+  if (p.fix_phase == 1 && (fseg <= 0 || fseg >= nseg)) return;
+  auto sstate = [&](const u32 *base, i64 seg) { return base + (seg * G::NG + G::GID) * G::NSMAX; };
   Ctx<K> c;
-  rx_ctx_init<G>(p, c, acc);
+  rx_ctx_init<G>(p, c, acc, lb);
   u32 pl[8][K];
   u32 xr[K][8];
   u32 *tru = sst, *old = sst + M, *t1 = sst + 2 * M, *t2 = sst + 3 * M;
   u32 fold[G::NR * K];
   c.fold = p.match_total ? fold : nullptr;
-  for (int s = (int)c.lane; s < NS; s += 32) {
-    tru[s] = p.st_in ? p.st_in[G::SBASE + s] : 0u;
-    old[s] = (p.mode == 2 && p.st_assumed) ? p.st_assumed[G::SBASE + s] : 0u;
-  }
-  __syncwarp();
-  for (i64 seg = 0; seg < nseg; ++seg) {
-    const i64 w_begin = seg * p.sw;
-    const i64 w_end = w_begin + p.sw < nwin ? w_begin + p.sw : nwin;
-    if (p.mode == 1) {
-      // the state pass 1 assumed for this segment
-      for (int s = (int)c.lane; s < NS; s += 32) old[s] = seg == 0 ? (p.st_in ? p.st_in[G::SBASE + s] : 0u) : 0u;
-      __syncwarp();
-    }
+  // re-run windows [w0, w1) with both states (old: the state the applied
+  // results assumed, subtracted; tru: the true state, added) until the two
+  // runs' states agree; returns whether they did
+  auto walk = [&](i64 w0, i64 w1) -> bool {
     bool conv = rx_state_eq(tru, old, NS, c.lane);
-    for (i64 w = w_begin; w < w_end && !conv; ++w) {
+    for (i64 w = w0; w < w1 && !conv; ++w) {
       const i64 cstart = w * Bw;
       const i64 fword = cstart - Lw;
       c.cw = (u32)((len_words - cstart) < Bw ? (len_words - cstart) : Bw);
@@ -668,10 +729,79 @@ DEV void rx_fixup_group(const RxParams &p, u64 *acc, u32 *sst) {
       rx_state_copy(tru, t2, NS, c.lane);
       conv = rx_state_eq(tru, old, NS, c.lane);
     }
+    return conv;
+  };
+  if (p.mode == 1 && p.fix_phase == 1) {
+    // phase 1 (one warp per (group, segment), all in parallel): pass 1 ran
+    // segment fseg from a zero state; its true incoming state is taken to be
+    // pass 1's end state of segment fseg-1 -- right unless that segment
+    // itself did not converge here, which is flagged (seg_nc) for phase 2
+    const u32 *src = sstate(p.seg_state, fseg - 1);
+    for (int s = (int)c.lane; s < NS; s += 32) {
+      tru[s] = src[s];
+      old[s] = 0u;
+    }
+    __syncwarp();
+    if (rx_state_eq(tru, old, NS, c.lane)) return;
+    const i64 w_begin = fseg * p.sw;
+    const i64 w_end = w_begin + p.sw < nwin ? w_begin + p.sw : nwin;
+    if (!walk(w_begin, w_end)) {
+      u32 *dst = p.seg_fix + (fseg * G::NG + G::GID) * G::NSMAX;
+      for (int s = (int)c.lane; s < NS; s += 32) dst[s] = tru[s];
+      if (c.lane == 0) p.seg_nc[fseg * G::NG + G::GID] = 1u;
+    }
+    rx_flush<G>(p, c);
+    return;
+  }
+  if (p.mode == 1 && p.fix_phase == 2) {
+    // phase 2 (one warp per group, serial over segments): only groups with a
+    // segment that did not converge in phase 1.  The results applied so far
+    // for segment s assume incoming A(s) = pass 1's end of s-1 (st_in for
+    // s = 0); walk from the true state T where T != A(s).
+    bool any = false;
+    for (i64 i = c.lane; i < nseg; i += 32) any = any || p.seg_nc[i * G::NG + G::GID] != 0u;
+    if (!__any_sync(RX_FULL, any)) return;
+    for (int s = (int)c.lane; s < NS; s += 32) tru[s] = p.st_in ? p.st_in[G::SBASE + s] : 0u;
+    __syncwarp();
+    for (i64 seg = 0; seg < nseg; ++seg) {
+      const u32 *a = seg == 0 ? nullptr : sstate(p.seg_state, seg - 1);
+      for (int s = (int)c.lane; s < NS; s += 32) old[s] = a ? a[s] : (p.st_in ? p.st_in[G::SBASE + s] : 0u);
+      __syncwarp();
+      const i64 w_begin = seg * p.sw;
+      const i64 w_end = w_begin + p.sw < nwin ? w_begin + p.sw : nwin;
+      if (walk(w_begin, w_end)) {
+        // converged: the applied run's end state stands
+        const bool nc = p.seg_nc[seg * G::NG + G::GID] != 0u;
+        const u32 *e = nc ? sstate(p.seg_fix, seg) : sstate(p.seg_state, seg);
+        for (int s = (int)c.lane; s < NS; s += 32) tru[s] = e[s];
+        __syncwarp();
+      }
+    }
+    if (p.st_out)
+      for (int s = (int)c.lane; s < NS; s += 32) p.st_out[G::SBASE + s] = tru[s];
+    rx_flush<G>(p, c);
+    return;
+  }
+  // serial form (rematch, mode 2; and mode 1 with fix_phase 0): one warp
+  // walks the segments in order carrying the true state
+  for (int s = (int)c.lane; s < NS; s += 32) {
+    tru[s] = p.st_in ? p.st_in[G::SBASE + s] : 0u;
+    old[s] = (p.mode == 2 && p.st_assumed) ? p.st_assumed[G::SBASE + s] : 0u;
+  }
+  __syncwarp();
+  for (i64 seg = 0; seg < nseg; ++seg) {
+    const i64 w_begin = seg * p.sw;
+    const i64 w_end = w_begin + p.sw < nwin ? w_begin + p.sw : nwin;
+    if (p.mode == 1) {
+      // the state pass 1 assumed for this segment
+      for (int s = (int)c.lane; s < NS; s += 32) old[s] = seg == 0 ? (p.st_in ? p.st_in[G::SBASE + s] : 0u) : 0u;
+      __syncwarp();
+    }
+    const bool conv = walk(w_begin, w_end);
     if (conv) {
       if (p.mode == 2) break;  // identical to the caller's run from here on
       // from here on pass 1's result stands: take its segment end state
-      const u32 *src = p.seg_state + (seg * G::NG + G::GID) * G::NSMAX;
+      const u32 *src = sstate(p.seg_state, seg);
       for (int s = (int)c.lane; s < NS; s += 32) tru[s] = src[s];
       __syncwarp();
     }
@@ -715,21 +845,18 @@ DEV u32 rx_pf_x(u32 w0, u32 w1, u32 w2, u32 w3, u32 w4, u32 w5, int r) {
 // the 4 bytes ending there (xa) and the 4 bytes after them (xc); the gram
 // ends d = 0..3 bytes later and is x(d) = funnel(xa, xc, 8d).  It is recorded
 // in the block of the bigram's end (inside the gram, hence inside every
-// window frame that contains the gram).
-DEV void rx_pf_record(const RxParams &p, const u32 *T, u32 *gt, u32 *blc, unsigned short *blf, u32 fid, int b) {
-  bool dup = false;
-  const u32 n0 = *(volatile u32 *)&blc[b];
-  for (u32 j = 0; j < n0 && j < 15u; ++j)
-    if (*(volatile unsigned short *)&blf[b * 15 + j] == (unsigned short)fid) dup = true;
-  if (dup) return;
-  const u32 slot = atomicAdd(&blc[b], 1u);
-  if (slot < 15u) blf[b * 15 + slot] = (unsigned short)fid;
+// window frame that contains the gram): the (group, member mask) pairs of the
+// factor are ORed into the tile's shared per-(group, block) member masks.
+DEV void rx_pf_record(const RxParams &p, const u32 *T, u32 *sm, u32 fid, int b) {
   const u32 f1 = T[p.pf_o_fgoff + fid + 1];
-  for (u32 j = T[p.pf_o_fgoff + fid]; j < f1; ++j) atomicOr(&gt[T[p.pf_o_fgent + 2 * j]], 1u << b);
+  for (u32 j = T[p.pf_o_fgoff + fid]; j < f1; ++j) {
+    u32 *a = &sm[T[p.pf_o_fgent + 2 * j] * 32u + (u32)b];
+    const u32 m = T[p.pf_o_fgent + 2 * j + 1];
+    if ((*(volatile u32 *)a & m) != m) atomicOr(a, m);
+  }
 }
 
-DEV void rx_pf_hit(const RxParams &p, const u32 *T, u32 *gt, u32 *blc, unsigned short *blf, u32 off, u32 xa,
-                   u32 xc, i64 tile_lo) {
+DEV void rx_pf_hit(const RxParams &p, const u32 *T, u32 *sm, u32 off, u32 xa, u32 xc, i64 tile_lo) {
   const u32 bg = xa >> 16, wi = bg >> 5, bit = bg & 31u;
   const u32 idx = T[2048 + wi] + __popc(T[wi] & ((1u << bit) - 1u));
   u32 shapes = T[4096 + idx];
@@ -749,13 +876,13 @@ DEV void rx_pf_hit(const RxParams &p, const u32 *T, u32 *gt, u32 *blc, unsigned 
     for (;;) {
       const u32 tag = H[2 * h + 1];
       if (tag == 0u) break;
-      if (H[2 * h] == key && ((tag >> 1) & 127u) == sh) rx_pf_record(p, T, gt, blc, blf, tag >> 8, b);
+      if (H[2 * h] == key && ((tag >> 1) & 127u) == sh) rx_pf_record(p, T, sm, tag >> 8, b);
       h = (h + 1u) & hmask;
     }
   }
 }
 
-// smem: [tables (if they fit) | gt NG | blc 32 | blf 32 x 15 u16 | per-warp hit queues 32 x 3]
+// smem: [tables (if they fit) | member masks NG x 32 | per-warp hit queues 32 x 3]
 DEV void rx_prefilter_run(const RxParams &p, int NG, bool tab_in_smem) {
   extern __shared__ __align__(16) u32 pf_smem[];
   const int tid = threadIdx.x, nt = blockDim.x;
@@ -764,16 +891,13 @@ DEV void rx_prefilter_run(const RxParams &p, int NG, bool tab_in_smem) {
   for (u32 i = tid; i < tw && i < p.pf_words; i += nt) tab[i] = __ldg(&p.pf_tab[i]);
   // l1 + rank are always staged; the rest is read through T
   const u32 *T = tab_in_smem ? (const u32 *)tab : p.pf_tab;
-  u32 *gt = pf_smem + tw;
-  u32 *blc = gt + ((NG + 3) & ~3);
-  unsigned short *blf = reinterpret_cast<unsigned short *>(blc + 32);
-  u32 *wq = blc + 32 + 240 + 96 * (tid >> 5);  // per-warp hit queue: 32 x {off, xa, xc}
+  u32 *sm = pf_smem + tw;                     // [NG][32 blocks] member masks
+  u32 *wq = sm + 32 * NG + 96 * (tid >> 5);  // per-warp hit queue: 32 x {off, xa, xc}
   const u32 lane = rx_lane();
   const i64 span = p.avail_hi - p.avail_lo;
   const i64 ntiles = (span + RX_PF_TILE - 1) / RX_PF_TILE;
   for (i64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
-    for (int i = tid; i < NG; i += nt) gt[i] = 0u;
-    if (tid < 32) blc[tid] = 0u;
+    for (int i = tid; i < 32 * NG; i += nt) sm[i] = 0u;
     __syncthreads();
     const i64 tile_lo = p.avail_lo + t * RX_PF_TILE;
     for (int j = 0; j < RX_PF_TILE / 16; j += nt) {
@@ -821,7 +945,7 @@ DEV void rx_prefilter_run(const RxParams &p, int NG, bool tab_in_smem) {
         }
         if (qn == 32u || (bal == 0u && qn > 0u)) {
           __syncwarp();
-          if (lane < qn) rx_pf_hit(p, T, gt, blc, blf, wq[3 * lane], wq[3 * lane + 1], wq[3 * lane + 2], tile_lo);
+          if (lane < qn) rx_pf_hit(p, T, sm, wq[3 * lane], wq[3 * lane + 1], wq[3 * lane + 2], tile_lo);
           __syncwarp();
           qn = 0;
         }
@@ -829,13 +953,14 @@ DEV void rx_prefilter_run(const RxParams &p, int NG, bool tab_in_smem) {
       }
     }
     __syncthreads();
-    for (int i = tid; i < NG; i += nt) p.pf_gbits[(i64)i * p.pf_ntiles + t] = gt[i];
-    for (int i = tid; i < 32 * 16; i += nt) {
-      const int b = i >> 4, e = i & 15;
-      const u32 n = blc[b];
-      if (n == 0u) continue;
-      const i64 gb = t * 32 + b;
-      p.pf_blist[gb * 16 + e] = e == 0 ? (unsigned short)(n > 0xffffu ? 0xffffu : n) : blf[b * 15 + e - 1];
+    // one warp per group: lane b holds block b's member mask; the group's
+    // tile word of block bits is their ballot
+    const i64 nblk = 32 * p.pf_ntiles;
+    for (int g = tid >> 5; g < NG; g += nt >> 5) {
+      const u32 v = sm[32 * g + lane];
+      const u32 bal = __ballot_sync(RX_FULL, v != 0u);
+      if (lane == 0) p.pf_gbits[(i64)g * p.pf_ntiles + t] = bal;
+      if (v) p.pf_mmask[(i64)g * nblk + t * 32 + lane] = v;
     }
     __syncthreads();
   }
@@ -865,7 +990,7 @@ DEV i64 rx_floor_div(i64 a, i64 b) { return a >= 0 ? a / b : -((-a + b - 1) / b)
 // and into which no state flows are skipped without loading a byte; the
 // others run only the members whose factor occurs in the frame, that carry
 // state, or that have no factor (G::ALWAYS).
-template <class G> DEV void rx_run_segment_pf(const RxParams &p, int seg, u64 *acc, u32 *sst) {
+template <class G> DEV void rx_run_segment_pf(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *lb) {
   constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS;
   const i64 len_words = rx_div_up(p.len, 32);
   const i64 nwin = rx_div_up(len_words, Bw);
@@ -873,7 +998,7 @@ template <class G> DEV void rx_run_segment_pf(const RxParams &p, int seg, u64 *a
   const bool live = w_begin < nwin || seg == 0;
   const i64 w_end = !live ? w_begin : (w_begin + p.sw < nwin ? w_begin + p.sw : nwin);
   Ctx<K> c;
-  rx_ctx_init<G>(p, c, acc);
+  rx_ctx_init<G>(p, c, acc, lb);
   u32 pl[8][K];
   u32 xr[K][8];
   u32 *st = sst, *nst = sst + G::NSMAX;
@@ -933,24 +1058,12 @@ template <class G> DEV void rx_run_segment_pf(const RxParams &p, int seg, u64 *a
         continue;
       }
     }
-    // members whose factor occurs in one of the frame's blocks
+    // members whose factor occurs in one of the frame's blocks (lane i
+    // looks at block b0 + i; a frame spans a few blocks)
+    const u32 *mm = p.pf_mmask + (i64)G::GID * 32 * p.pf_ntiles;
     u32 mine = 0u;
-    for (i64 b = b0; b <= b1; ++b) {
-      if (!((gb[b >> 5] >> (b & 31)) & 1u)) continue;
-      const unsigned short *L = p.pf_blist + b * 16;
-      const u32 n = L[0];
-      if (n > 15u) {
-        mine = RX_FULL;
-        break;
-      }
-      if (c.lane < n) {
-        const u32 fid = L[1 + c.lane];
-        const u32 *fo = p.pf_tab + p.pf_o_fgoff, *fe = p.pf_tab + p.pf_o_fgent;
-        const u32 f1 = __ldg(&fo[fid + 1]);
-        for (u32 j = __ldg(&fo[fid]); j < f1; ++j)
-          if (__ldg(&fe[2 * j]) == (u32)G::GID) mine |= __ldg(&fe[2 * j + 1]);
-      }
-    }
+    for (i64 b = b0 + c.lane; b <= b1; b += 32)
+      if ((gb[b >> 5] >> (b & 31)) & 1u) mine |= mm[b];
     const u32 rmask = __reduce_or_sync(RX_FULL, mine);
     if (p.stats && c.lane == 0) {
       // [0] active windows [1] of them only for carried state [2] members hit
@@ -978,6 +1091,141 @@ template <class G> DEV void rx_run_segment_pf(const RxParams &p, int seg, u64 *a
     if (!lockstep) ++w;
   }
   if (lockstep && step > 0) __syncthreads();
+  if (!live) return;
+  if (NS > 0) {
+    u32 *dst = p.seg_state + ((i64)seg * G::NG + G::GID) * G::NSMAX;
+    for (int s = (int)c.lane; s < NS; s += 32) dst[s] = st[s];
+    if (p.st_out && w_end == nwin)
+      for (int s = (int)c.lane; s < NS; s += 32) p.st_out[G::SBASE + s] = st[s];
+  }
+  rx_flush<G>(p, c);
+}
+
+// Sparse pass 1 with a one-window lookahead (the default): while the body
+// of window w runs, the bytes of the window expected next -- w + 1 if state
+// flows into w (it usually flows on), else the next window whose frame holds
+// a factor of the group -- are already on their way into a per-warp shared
+// buffer by a TMA bulk copy.  A wrong guess costs a synchronous global load;
+// the window order and the set of windows run are exactly those of
+// rx_run_segment_pf (running an extra window with no state and no factor is
+// harmless: its output and state are zero).
+template <class G>
+DEV void rx_run_segment_pf_staged(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *tbuf, u64 *bar,
+                                  unsigned char *lb) {
+  constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS;
+  constexpr u32 WB = 1024u * K;
+  const i64 len_words = rx_div_up(p.len, 32);
+  const i64 nwin = rx_div_up(len_words, Bw);
+  const i64 w_begin = (i64)seg * p.sw;
+  const bool live = w_begin < nwin || seg == 0;
+  const i64 w_end = !live ? w_begin : (w_begin + p.sw < nwin ? w_begin + p.sw : nwin);
+  Ctx<K> c;
+  rx_ctx_init<G>(p, c, acc, lb);
+  u32 pl[8][K];
+  u32 xr[K][8];
+  u32 *st = sst, *nst = sst + G::NSMAX;
+  for (int s = (int)c.lane; s < NS; s += 32) st[s] = (seg == 0 && p.st_in) ? p.st_in[G::SBASE + s] : 0u;
+  if (c.lane == 0) rx_mbar_init(bar, 1);
+  __syncwarp();
+  const RxRange ir = rx_interior(p);
+  const u32 *gb = p.pf_gbits + (i64)G::GID * p.pf_ntiles;
+  const u32 *mm = p.pf_mmask + (i64)G::GID * 32 * p.pf_ntiles;
+  auto frame_blocks = [&](i64 w, i64 &b0, i64 &b1) {
+    i64 flo = (w * Bw - Lw) * 32, fhi = flo + 1024 * K;
+    if (flo < p.avail_lo) flo = p.avail_lo;
+    if (fhi > p.avail_hi) fhi = p.avail_hi;
+    if (fhi <= flo) fhi = flo + 1;
+    b0 = (flo - p.avail_lo) >> 10;
+    b1 = (fhi - 1 - p.avail_lo) >> 10;
+  };
+  i64 bmax = 0;
+  if (w_begin < w_end) {
+    i64 t0;
+    frame_blocks(w_end - 1, t0, bmax);
+  }
+  auto pending = [&](const u32 *a) -> bool {
+    if (NS == 0) return false;
+    bool any = false;
+    for (int s = (int)c.lane; s < NS; s += 32) any = any || a[s] != 0u;
+    return __any_sync(RX_FULL, any);
+  };
+  // first window >= w whose frame holds a factor of the group (w_end if none)
+  auto next_hit = [&](i64 w) -> i64 {
+    if (w >= w_end) return w_end;
+    if (G::ALWAYS != 0u) return w;
+    i64 b0, b1;
+    frame_blocks(w, b0, b1);
+    const i64 b = rx_pf_next(gb, b0, bmax, c.lane);
+    if (b > bmax) return w_end;
+    if (b <= b1) return w;
+    const i64 pos = p.avail_lo + b * RX_PF_BLK;
+    const i64 wn = rx_floor_div(rx_floor_div(pos, 32) + Lw - 32 * K, Bw) + 1;
+    const i64 r = wn > w + 1 ? wn : w + 1;
+    return r < w_end ? r : w_end;
+  };
+  i64 staged = -1;  // window whose bytes are in flight / in tbuf (-1: none)
+  u32 phase = 0;
+  auto stage = [&](i64 w) {
+    const i64 f = w * Bw - Lw;
+    if (w < w_end && f >= ir.lo && f + 32 * K <= ir.hi) {
+      __syncwarp();
+      if (c.lane == 0) rx_bulk_load(tbuf, p.in + f * 32, WB, bar);
+      staged = w;
+    }
+  };
+  auto retire = [&]() {  // wait for the copy in flight (keeps the mbarrier phase in step)
+    rx_mbar_wait(bar, phase);
+    phase ^= 1u;
+    staged = -1;
+  };
+  i64 w = pending(st) ? w_begin : next_hit(w_begin);
+  if (w < w_end) stage(w);
+  while (w < w_end) {
+    const bool pend_in = pending(st);
+    if (p.stats && c.lane == 0) atomicAdd(&p.stats[3], 1ull);
+    const i64 fword = w * Bw - Lw;
+    if (staged == w) {
+      retire();
+      const uint4 *q = reinterpret_cast<const uint4 *>(tbuf + c.lane * (32u * K));
+#pragma unroll
+      for (int k = 0; k < K; ++k) {
+        const uint4 a0 = q[2 * k], a1 = q[2 * k + 1];
+        xr[k][0] = a0.x; xr[k][1] = a0.y; xr[k][2] = a0.z; xr[k][3] = a0.w;
+        xr[k][4] = a1.x; xr[k][5] = a1.y; xr[k][6] = a1.z; xr[k][7] = a1.w;
+      }
+    } else {
+      if (staged >= 0 && staged < w) retire();  // a stale guess: drain it
+      rx_fetch<K>(p, ir, c.lane, xr, fword);
+    }
+    // guess the next window and start its copy before the body runs
+    if (staged < 0) {
+      const i64 guess = pend_in ? w + 1 : next_hit(w + 1);
+      stage(guess);
+    }
+    i64 b0, b1;
+    frame_blocks(w, b0, b1);
+    u32 mine = 0u;
+    for (i64 b = b0 + c.lane; b <= b1; b += 32)
+      if ((gb[b >> 5] >> (b & 31)) & 1u) mine |= mm[b];
+    const u32 rmask = __reduce_or_sync(RX_FULL, mine);
+    if (p.stats && c.lane == 0) {
+      atomicAdd(&p.stats[0], 1ull);
+      if (rmask == 0u) atomicAdd(&p.stats[1], 1ull);
+      atomicAdd(&p.stats[2], (u64)__popc(rmask));
+    }
+    c.cw = (u32)((len_words - w * Bw) < Bw ? (len_words - w * Bw) : Bw);
+    c.word0 = fword;
+    rx_unpack<K>(p, ir, c, xr, pl, fword);
+    rx_commit_mask(p, ir, c, Lw, fword);
+    if (NS > 0) rx_state_zero(nst, NS, c.lane);
+    G::body(c, pl, st, nst, rmask);
+    u32 *t = st;
+    st = nst;
+    nst = t;
+    __syncwarp();
+    w = pending(st) ? w + 1 : next_hit(w + 1);
+  }
+  if (staged >= 0) retire();
   if (!live) return;
   if (NS > 0) {
     u32 *dst = p.seg_state + ((i64)seg * G::NG + G::GID) * G::NSMAX;

@@ -63,6 +63,9 @@ enum class Op : uint8_t {
   Loop,    // while-fixpoint of Fig. 2e / Listing 3: acc = lfp(seeds U body(acc))
   Fr,      // the frontier placeholder inside a Loop body
   Guard,   // zero-block-skipping region (Sec. 6): value = region result, or 0 if any(cond)==0
+  Lit,     // literal run: out[p] = in[p-k] & (input[p-k+1..p] == lits[cc]) -- exactly the chain
+           // v_j = Adv(v_{j-1}, 1) & CC(lits[cc][j]) (Fig. 2b/2c) for j = 1..k, evaluated by
+           // confirming the (sparse) marker positions byte by byte
 };
 
 struct Node {
@@ -89,6 +92,7 @@ struct RegexIR {
   std::vector<Node> nodes;
   std::vector<Block> blocks;  // blocks[0] = top level
   std::vector<ByteSet> sets;
+  std::vector<std::string> lits;  // Lit: literal byte strings (no 0x00 byte)
   int out = -1;               // result node (top level) of a single-regex IR
   std::vector<int> outs;      // result nodes of a cluster IR (one per member regex; outs[0] == out)
   int nslots = 0;
@@ -105,6 +109,11 @@ struct LowerOptions {
   // unanchored chain (with the prefilter the regex only runs where its
   // factor occurs, and an unguarded head can be shared by a factor cluster)
   bool lead_noguard = false;
+  // literal runs: after `lit_after` single-byte items of a chain (the marker
+  // stream is then sparse), a run of >= lit_min further single-byte items
+  // becomes one Lit node; lit_min <= 0: never
+  int lit_after = 3;
+  int lit_min = 2;
 };
 
 // Lower one parsed regex to IR (non-empty, unanchored match ends).
@@ -175,6 +184,7 @@ struct CompiledSet {
 // into one module with nvJitLink.
 std::string emit_group_unit(CompiledSet &cs, int gi);
 std::string emit_kernel_unit(CompiledSet &cs);
+int lit_scratch_bytes(const CompiledSet &cs);  // per-warp shared bytes of the literal-run scratch
 bool plan_groups(CompiledSet &cs, int group_size, int force_K, std::string &why);
 void build_prefilter(CompiledSet &cs);
 // Partition each group's members into clusters (same factor, or no factor)

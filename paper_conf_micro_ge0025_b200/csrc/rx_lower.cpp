@@ -47,6 +47,7 @@ struct Lowerer {
   std::vector<int> loops;                   // enclosing loop nodes
   std::vector<std::map<Key, int>> cse;      // scoped hash-consing
   std::map<std::vector<uint64_t>, int> set_ix;
+  std::map<std::string, int> lit_ix;
   int zero = -1, ones = -1;
   size_t since_guard = 0;
 
@@ -132,6 +133,75 @@ struct Lowerer {
     return mk(Op::CC, -1, -1, 0, ix);
   }
 
+  int LIT(int m, const std::string &s) {
+    if (is(m, Op::Zero)) return zero;
+    int ix;
+    auto f = lit_ix.find(s);
+    if (f == lit_ix.end()) {
+      ix = (int)ir.lits.size();
+      ir.lits.push_back(s);
+      lit_ix[s] = ix;
+    } else {
+      ix = f->second;
+    }
+    return mk(Op::Lit, m, -1, (int)s.size(), ix);
+  }
+  // a Once item matching exactly one byte value, not 0x00 (the Lit confirm
+  // compares raw bytes; 0x00 is also the padding beyond the stream)
+  static bool single_byte(const Item &it, int &c) {
+    ByteSet s;
+    if (it.mode != Item::Once || !single_set(*it.ast, s) || s.count() != 1) return false;
+    for (int b = 1; b < 256; ++b)
+      if (s.has(b)) {
+        c = b;
+        return true;
+      }
+    return false;
+  }
+
+  int ADVK(int m, int k) {
+    if (k == 0) return m;
+    if (is(m, Op::Zero)) return zero;
+    if (is(m, Op::Ones)) return ones;
+    return mk(Op::Adv, m, -1, k);
+  }
+  // Cr_t = positions q whose t bytes (q-t, q] are all in class C, by
+  // doubling: Cr_{x+y} = Cr_x & Adv(Cr_y, x) (Fig. 2d's bounded repetition
+  // unrolls this one byte at a time; the result is the same stream)
+  int CRUN(int C, int t) {
+    std::vector<int> pw = {C};  // pw[j] = Cr_{2^j}
+    while ((1 << pw.size()) <= t) {
+      int j = (int)pw.size() - 1;
+      pw.push_back(AND(pw[j], ADVK(pw[j], 1 << j)));
+    }
+    int res = -1, len = 0;
+    for (int j = (int)pw.size() - 1; j >= 0; --j)
+      if ((t >> j) & 1) {
+        res = res < 0 ? pw[j] : AND(res, ADVK(pw[j], len));
+        len += 1 << j;
+      }
+    return res;
+  }
+  // E(C{lo,hi}, M), C a single class, hi >= 0: the non-empty ends q with
+  // some p in M, max(lo,1) <= q-p <= hi and bytes (p, q] all in C.  Exact
+  // distance a = max(lo,1) first (Y), then the reach S_t(Y) of up to t more
+  // C bytes extended by doubling: S_{t+b} = S_t | (Adv(S_t, b) & Cr_b) for
+  // b <= t+1.  O(log hi) operations instead of the (hi-lo) optional items of
+  // Fig. 2d; the result is the same stream (tests: brute force over {n,m}).
+  int E_crep(const ByteSet &cs, int lo, int hi, int M) {
+    int C = CC(cs);
+    int a = std::max(lo, 1);
+    if (hi < a) return zero;
+    int Y = is(M, Op::Ones) ? CRUN(C, a) : AND(ADVK(M, a), CRUN(C, a));
+    int S = Y;
+    for (int t = 0; t < hi - a && !is(S, Op::Zero);) {
+      int b = std::min(t + 1, hi - a - t);
+      S = OR(S, AND(ADVK(S, b), CRUN(C, b)));
+      t += b;
+    }
+    return S;
+  }
+
   // --- E(R, M) -------------------------------------------------------------
   static const Ast *single_set(const Ast &a, ByteSet &out) {
     // A sub-expression that matches exactly one byte from a set: Set, or
@@ -170,6 +240,18 @@ struct Lowerer {
       case AK::Rep: {
         const Ast &kid = *r.kids[0];
         if (r.hi == 0) return zero;
+        {
+          ByteSet cs;
+          if (loops.empty() && single_set(kid, cs) && !cs.empty()) {
+            if (r.hi >= 0 && (r.hi - std::max(r.lo, 1) >= 3 || r.lo >= 5)) return E_crep(cs, r.lo, r.hi, M);
+            if (r.hi < 0 && r.lo >= 6) {
+              // C{n,} = C{n-1} C+ : the fixed part by doubling, then MatchStar
+              int C = CC(cs);
+              int Y = is(M, Op::Ones) ? CRUN(C, r.lo - 1) : AND(ADVK(M, r.lo - 1), CRUN(C, r.lo - 1));
+              return E_plus(kid, Y);
+            }
+          }
+        }
         std::vector<Item> items;
         if (r.hi < 0) {
           for (int i = 0; i + 1 < r.lo; ++i) items.push_back({&kid, Item::Once});
@@ -198,7 +280,7 @@ struct Lowerer {
 
   // Concatenation items[j..] after a prefix whose (possibly empty) end
   // markers are P and whose non-empty end markers are N.
-  int E_cat(const std::vector<Item> &items, size_t j, int P, int N, bool guarded = false) {
+  int E_cat(const std::vector<Item> &items, size_t j, int P, int N, bool guarded = false, int single_run = 0) {
     // leading run of single-class items of an unanchored chain: unguarded
     // with opt.lead_noguard (LowerOptions)
     size_t lead = 0;
@@ -206,6 +288,7 @@ struct Lowerer {
       ByteSet tmp;
       while (lead < items.size() && items[lead].mode == Item::Once && single_set(*items[lead].ast, tmp)) ++lead;
     }
+    // single_run: single-byte items just consumed by this chain
     for (; j < items.size(); ++j) {
       // Zero-block-skipping guard (Sec. 6): P is a zero-path
       // head -- if P is all-zero in a window, everything downstream in this
@@ -222,14 +305,33 @@ struct Lowerer {
         ir.n_guards++;
         int sb = push_block();
         since_guard = 0;
-        int res = E_cat(items, j, P, N, true);
+        int res = E_cat(items, j, P, N, true, single_run);
         pop_block();
         ir.nodes[gid].sub = sb;
         ir.nodes[gid].res = res;
         if (is(res, Op::Zero)) return zero;
         return gid;
       }
+      // literal run (LowerOptions::lit_after / lit_min): one Lit node
+      int cb = 0;
+      if (opt.lit_min > 0 && loops.empty() && single_run >= opt.lit_after && !is(P, Op::Ones) &&
+          single_byte(items[j], cb)) {
+        std::string s;
+        size_t r = j;
+        for (int c2 = 0; r < items.size() && single_byte(items[r], c2); ++r) s += (char)c2;
+        if ((int)s.size() >= opt.lit_min) {
+          P = N = LIT(P, s);
+          single_run += (int)s.size();
+          j = r - 1;
+          if (is(P, Op::Zero)) return zero;
+          continue;
+        }
+      }
       const Item &it = items[j];
+      {
+        int c3 = 0;
+        single_run = single_byte(it, c3) ? single_run + 1 : 0;
+      }
       int e = E_item(it, P);
       if (item_nullable(it)) {
         int nP = OR(e, P);
@@ -389,6 +491,11 @@ static void margins_block(RegexIR &ir, int block, int &slot) {
         n.rb = std::max(rb(n.a) - n.k, 0);
         n.depth = dp(n.a) + 1;
         break;
+      case Op::Lit:  // = k advances by one (and ANDs with classes)
+        n.lb = lb(n.a) + n.k;
+        n.rb = std::max(rb(n.a) - n.k, 0);
+        n.depth = dp(n.a) + 1;
+        break;
       case Op::Look:
         n.lb = std::max(lb(n.a) - n.k, 0);
         n.rb = rb(n.a) + n.k;
@@ -440,7 +547,7 @@ bool analyze_regex(RegexIR &ir, std::string &why) {
 
 std::string dump_ir(const RegexIR &ir) {
   static const char *names[] = {"zero", "ones", "cc", "and", "or", "xor", "andn", "adv", "look",
-                                "mstar", "loop", "fr", "guard"};
+                                "mstar", "loop", "fr", "guard", "lit"};
   std::ostringstream os;
   std::function<void(int, int)> blk = [&](int b, int ind) {
     for (int id : ir.blocks[b].nodes) {
@@ -450,6 +557,7 @@ std::string dump_ir(const RegexIR &ir) {
       if (n.b >= 0) os << " v" << n.b;
       if (n.op == Op::Adv || n.op == Op::Look) os << " k=" << n.k;
       if (n.op == Op::CC) os << " set#" << n.cc;
+      if (n.op == Op::Lit) os << " k=" << n.k << " lit#" << n.cc;
       os << "   [lb=" << n.lb << " rb=" << n.rb;
       if (n.slot >= 0) os << " slot=" << n.slot << " aw=" << n.aw;
       if (n.loop >= 0) os << " in-loop v" << n.loop;

@@ -183,6 +183,7 @@ bool nvrtc_compile(const std::string &src, int max_regs, bool use_cache, std::st
 struct RxModule {
   int g_begin = 0, g_end = 0;  // group range
   int ns_max = 1, nr_max = 1;
+  int lit_bytes = 0;  // per-warp literal-run scratch (rx_codegen.cpp lit_scratch_bytes)
   bool any_state = false;
   std::string source;
   std::vector<std::string> units;  // relocatable sm_100a cubins (groups + kernels)
@@ -228,7 +229,7 @@ const char *rx_program_source(const rx_program *p) { return p ? p->all_source.c_
 uint32_t rx_kernels_per_match(const rx_program *p) {
   uint32_t n = 0;
   if (p)
-    for (auto &m : p->mods) n += 1 + (m.any_state ? 1 : 0) + (p->cs.use_pf ? 1 : 0);
+    for (auto &m : p->mods) n += 1 + (m.any_state ? 2 : 0) + (p->cs.use_pf ? 1 : 0);
   return n;
 }
 const char *rx_program_info(const rx_program *p) { return p ? p->info.c_str() : ""; }
@@ -394,6 +395,7 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
     sbase += (uint32_t)g.nslots;
   }
   p->state_words = sbase;
+  mm.lit_bytes = rx::lit_scratch_bytes(p->cs);
   info << "prefilter: " << (p->cs.use_pf ? "on" : "off") << ", factors=" << p->cs.factors.size() << "\n";
   for (uint32_t i = 0; i < n_patterns; ++i) {
     const int f = p->cs.factor_of[i];
@@ -484,7 +486,7 @@ struct RxParamsHost {  // must mirror RxParams in rx_device.cuh
   unsigned int pf_hbits;
   int pf_tab_smem;
   unsigned int *pf_gbits;
-  unsigned short *pf_blist;
+  unsigned int *pf_mmask;
   long long pf_ntiles;
   int pf_on;
   int pf_aligned;
@@ -493,6 +495,9 @@ struct RxParamsHost {  // must mirror RxParams in rx_device.cuh
   unsigned long long *matches;
   unsigned long long match_cap;
   unsigned long long *match_total;
+  int fix_phase;
+  unsigned int *seg_fix;
+  unsigned int *seg_nc;
 };
 
 rx_status ensure_loaded(rx_program *p, int &device) {
@@ -557,10 +562,11 @@ rx_status launch(rx_program *p, RxModule &m, CUfunction f, long long blocks, int
   // must match the layout emitted in rx_codegen.cpp (accumulators | state |
   // TMA window staging | mbarriers); the fix-up kernel uses the first two
   const size_t wpb = (size_t)warps_per_block;
-  size_t bytes = wpb * 3 * m.nr_max * 8 + (((wpb * 4 * m.ns_max) + 3) & ~(size_t)3) * 4;
+  size_t bytes = wpb * 3 * m.nr_max * 8 + (((wpb * 4 * m.ns_max) + 3) & ~(size_t)3) * 4 + wpb * (size_t)m.lit_bytes;
   if (f == m.pass1) bytes += wpb * 4096 + wpb * 16;
   if (f == m.prefilter)
-    bytes = 4 * ((prm.pf_tab_smem ? ((prm.pf_words + 3) & ~3u) : 4096u) + (((m.g_end - m.g_begin) + 3) & ~3) + 32 + 240 + 96 * (size_t)warps_per_block);
+    bytes = 4 * ((prm.pf_tab_smem ? ((prm.pf_words + 3) & ~3u) : 4096u) + 32 * (size_t)(m.g_end - m.g_begin) +
+                 96 * (size_t)warps_per_block);
   unsigned smem = (unsigned)bytes;
   if (smem > 48 * 1024) d.FuncSetAttribute(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)smem);
   RxParamsHost local = prm;
@@ -679,7 +685,7 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
       const long long span = prm.avail_hi - prm.avail_lo;
       const long long ntiles = std::max<long long>(1, div_up(span, 32768));
       const size_t gb_bytes = (size_t)4 * (size_t)ntiles * (size_t)mg;
-      const size_t bl_bytes = (size_t)ntiles * 32 * 32;
+      const size_t bl_bytes = (size_t)4 * 32 * (size_t)ntiles * (size_t)mg;
       if (cudaMallocAsync(&pf_scratch, gb_bytes + bl_bytes + 256, stream) != cudaSuccess)
         return fail(RX_ENOMEM, "prefilter scratch");
       prm.pf_tab = (const unsigned int *)m.pf_mem;
@@ -688,9 +694,13 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
       prm.pf_o_fgoff = p->cs.pf.o_fgoff;
       prm.pf_o_fgent = p->cs.pf.o_fgent;
       prm.pf_hbits = p->cs.pf.hbits;
-      prm.pf_tab_smem = 4ull * prm.pf_words <= 160 * 1024 ? 1 : 0;
+      // shared memory: [table (or its 16 KiB bigram bitmap + rank) | NG x 32 member masks | hit queues]
+      const size_t fixed = 128ull * (size_t)mg + 6144;
+      prm.pf_tab_smem = 4ull * prm.pf_words + fixed <= 220 * 1024 ? 1 : 0;
+      if (!prm.pf_tab_smem && 16384 + fixed > 227 * 1024)
+        return fail(RX_ETOOBIG, "too many groups for the prefilter's shared member masks");
       prm.pf_gbits = (unsigned int *)pf_scratch;
-      prm.pf_blist = (unsigned short *)((char *)pf_scratch + ((gb_bytes + 255) & ~(size_t)255));
+      prm.pf_mmask = (unsigned int *)((char *)pf_scratch + ((gb_bytes + 255) & ~(size_t)255));
       prm.pf_ntiles = ntiles;
       prm.pf_on = 1;
       prm.pf_aligned = (((uintptr_t)(d_input - halo_left)) & 15) == 0 ? 1 : 0;
@@ -724,7 +734,28 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
     if (s != RX_OK) return s;
     if (m.any_state) {
       prm.mode = 1;
-      s = launch(p, m, m.fixup, div_up(mg, kFixupWarps), kFixupWarps, prm, stream);
+      const char *fe = getenv("RX_FIX_SERIAL");  // experiment knob: the one-warp-per-group serial fix-up
+      if (fe && *fe == '1') {
+        prm.fix_phase = 0;
+        s = launch(p, m, m.fixup, div_up(mg, kFixupWarps), kFixupWarps, prm, stream);
+      } else {
+        // phase 1: one warp per (group, segment) in parallel; phase 2: one
+        // warp per group, only where a segment's carry outlived it
+        void *fx = nullptr;
+        const size_t nc_bytes = 4ull * (size_t)nseg_max * (size_t)mg;
+        if (cudaMallocAsync(&fx, bytes + nc_bytes + 256, stream) != cudaSuccess) return fail(RX_ENOMEM, "fix-up scratch");
+        prm.seg_fix = (unsigned int *)fx;
+        prm.seg_nc = (unsigned int *)((char *)fx + ((bytes + 255) & ~(size_t)255));
+        cudaMemsetAsync(prm.seg_nc, 0, nc_bytes, stream);
+        prm.fix_phase = 1;
+        s = launch(p, m, m.fixup, div_up((long long)mg * nseg_max, kFixupWarps), kFixupWarps, prm, stream);
+        if (s == RX_OK) {
+          prm.fix_phase = 2;
+          s = launch(p, m, m.fixup, div_up(mg, kFixupWarps), kFixupWarps, prm, stream);
+        }
+        prm.fix_phase = 0;
+        cudaFreeAsync(fx, stream);
+      }
       if (s != RX_OK) return s;
       cudaFreeAsync(seg_state, stream);
     }

@@ -179,3 +179,25 @@ def test_match_list_equals_oracle_positions():
     assert int(out2["match_total"].cpu()[0]) == reg.size
     with pytest.raises(rx.RxError):
         prog.match_list(out2)
+
+
+def test_bounded_class_repeats_and_literal_runs():
+    # C{n,m} lowered by doubling (O(log m) steps) and literal runs confirmed
+    # byte by byte (Op::Lit) must give the chain's stream exactly: repeats
+    # of every shape, runs crossing lanes / windows, literals at frame edges
+    pats = [rb"ab[0-9]{0,7}x", rb"[a-c]{3,9}", rb"q[^\n]{5,40}z", rb"x[ab]{6,}y", rb"hello world literal run",
+            rb"[a-z]{1,64}", rb"abcdefghij", rb"a{4,16}", rb"zz[0-9a-f]{2}(?:%[0-9a-f]{2}){0,5}q",
+            rb"GET /index\.html HTTP/1\.[01]", rb"k[^\r\n]{0,64}\r\n", rb"[ab]{33,70}", rb"xyz.{0,100}uvw",
+            rb"(?:foo|bar)baz[0-9]{2,12}done"]
+    rng = np.random.default_rng(99)
+    alpha = np.frombuffer(b"abcxyz0123456789qk \n\r%fhelowrdGETHTP/.", dtype=np.uint8)
+    n = 300000
+    buf = bytearray(alpha[rng.integers(0, alpha.size, size=n)].tobytes())
+    plants = [b"hello world literal run", b"abcdefghij", b"GET /index.html HTTP/1.1", b"a" * 20, b"ab" * 40,
+              b"q" + b"w" * 30 + b"z", b"k" + b"m" * 64 + b"\r\n", b"xyz" + b"-" * 90 + b"uvw",
+              b"foobaz1234567done", b"zz0f%00%ab%ffq", b"x" + b"ab" * 10 + b"y"]
+    for at in list(range(1000, n - 200, 1023)) + [n - 30]:
+        s = plants[int(rng.integers(0, len(plants)))]
+        at = min(at, n - len(s))
+        buf[at:at + len(s)] = s
+    assert_parity(pats, bytes(buf))
