@@ -534,46 +534,80 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
     // state into the window run regardless
     // one out-of-line copy shared by pass 1 and both fix-up runs (code size,
     // NVRTC time; the call costs nothing next to the body)
-    os << "  static __device__ __noinline__ void body(Ctx<" << g.K << "> &c, const u32 (&pl)[8][" << g.K
-       << "], const u32 *st, u32 *nst, const u32 rmask) {\n";
-    os << "    (void)st; (void)nst; (void)rmask;\n";
-    os << "    const u32 lane = c.lane; const int cw = (int)c.cw; (void)cw;\n";
-    for (int k = 0; k < 8; ++k)
-      for (int i = 0; i < g.K; ++i) os << "    const u32 b" << k << "w" << i << " = pl[" << k << "][" << i << "];\n";
-    for (int i = 0; i < g.K; ++i) os << "    const u32 vmw" << i << " = c.vm[" << i << "];\n";
-    std::vector<std::map<TabKey, std::string>> ccs(1);
-    std::vector<std::map<std::vector<uint64_t>, std::string>> sets(1);
-    // one block per factor cluster: its unguarded (shared) head and guard
-    // tests (phase 1), then its guarded bodies (phase 2) if a guard fired
-    for (size_t ci = 0; ci < g.clusters.size(); ++ci) {
-      const Cluster &cl = g.clusters[ci];
-      RegexEmitter em(os, cl.ir, g.K, (int)ci, cl.slot_base, ccs, sets);
-      em.out_member = cl.members;
-      em.lit_pool = "rx_litb_" + std::to_string(gi);
-      em.lit_off = lit_off[ci];
-      std::string run;
-      if (cl.always) {
-        run = "true";
-      } else {
-        uint32_t mm = 0;
-        for (int m : cl.members) mm |= 1u << m;
-        run = "(rmask & " + std::to_string(mm) + "u) != 0u";
-        if (cl.ir.nslots > 0) {
-          std::string pend;
-          for (int sl = 0; sl < cl.ir.nslots; ++sl) pend += (sl ? " | " : "") + em.st(sl);
-          run += " || ((" + pend + ") != 0u)";
+    // The group's program: body() runs every factor cluster in one
+    // out-of-line function (shared by pass 1 and both fix-up runs), with
+    // the CC networks CSE'd across the clusters.  With cluster-major code
+    // generation (RX_CMAJOR_GEN=1, an experiment: DESIGN.md "Scheduling")
+    // each cluster also gets its own function cb<ci> that pass 1 runs over
+    // consecutive windows.
+    const int NC = (int)g.clusters.size();
+    const char *cmg = getenv("RX_CMAJOR_GEN");
+    const bool gen_cm = cmg && *cmg == '1';
+    std::vector<uint32_t> cmask(NC, 0u);
+    for (int ci = 0; ci < NC; ++ci)
+      for (int m : g.clusters[ci].members) cmask[ci] |= 1u << m;
+    auto emit_fn = [&](const std::string &name, int c0, int c1) {
+      os << "  static __device__ __noinline__ void " << name << "(Ctx<" << g.K << "> &c, const u32 (&pl)[8][" << g.K
+         << "], const u32 *st, u32 *nst, const u32 rmask) {\n";
+      os << "    (void)st; (void)nst; (void)rmask;\n";
+      os << "    const u32 lane = c.lane; const int cw = (int)c.cw; (void)cw; (void)lane;\n";
+      for (int k = 0; k < 8; ++k)
+        for (int i = 0; i < g.K; ++i)
+          os << "    const u32 b" << k << "w" << i << " = pl[" << k << "][" << i << "]; (void)b" << k << "w" << i << ";\n";
+      for (int i = 0; i < g.K; ++i) os << "    const u32 vmw" << i << " = c.vm[" << i << "]; (void)vmw" << i << ";\n";
+      std::vector<std::map<TabKey, std::string>> ccs(1);
+      std::vector<std::map<std::vector<uint64_t>, std::string>> sets(1);
+      for (int ci = c0; ci < c1; ++ci) {
+        const Cluster &cl = g.clusters[ci];
+        RegexEmitter em(os, cl.ir, g.K, ci, cl.slot_base, ccs, sets);
+        em.out_member = cl.members;
+        em.lit_pool = "rx_litb_" + std::to_string(gi);
+        em.lit_off = lit_off[ci];
+        std::string run;
+        if (cl.always) {
+          run = "true";
+        } else {
+          run = "(rmask & " + std::to_string(cmask[ci]) + "u) != 0u";
+          if (cl.ir.nslots > 0) {
+            std::string pend;
+            for (int sl = 0; sl < cl.ir.nslots; ++sl) pend += (sl ? " | " : "") + em.st(sl);
+            run += " || ((" + pend + ") != 0u)";
+          }
         }
-      }
-      os << "    if (" << run << ") {\n";
-      em.push();
-      std::string need = em.emit_phase1();
-      if (!need.empty()) {
-        os << "    if (" << need << ") {\n";
-        em.emit_phase2();
+        // one block per factor cluster: its unguarded (shared) head and guard
+        // tests (phase 1), then its guarded bodies (phase 2) if a guard fired
+        os << "    if (" << run << ") {\n";
+        em.push();
+        std::string need = em.emit_phase1();
+        if (!need.empty()) {
+          os << "    if (" << need << ") {\n";
+          em.emit_phase2();
+          os << "    }\n";
+        }
+        em.pop();
         os << "    }\n";
       }
-      em.pop();
-      os << "    }\n";
+      os << "  }\n";
+    };
+    emit_fn("body", 0, NC);
+    if (gen_cm)
+      for (int ci = 0; ci < NC; ++ci) emit_fn("cb" + std::to_string(ci), ci, ci + 1);
+    os << "  static constexpr int NC = " << (gen_cm ? NC : 0) << ";\n";
+    os << "  static DEV u32 cmask(int ci) {\n    switch (ci) {\n";
+    for (int ci = 0; ci < NC; ++ci) os << "      case " << ci << ": return " << cmask[ci] << "u;\n";
+    os << "      default: return 0u;\n    }\n  }\n";
+    os << "  static DEV bool calways(int ci) {\n    switch (ci) {\n";
+    for (int ci = 0; ci < NC; ++ci) os << "      case " << ci << ": return " << (g.clusters[ci].always ? "true" : "false") << ";\n";
+    os << "      default: return false;\n    }\n  }\n";
+    os << "  static DEV int cslot(int ci) {  // first state slot of cluster ci (ci = NC: total)\n    switch (ci) {\n";
+    for (int ci = 0; ci < NC; ++ci) os << "      case " << ci << ": return " << g.clusters[ci].slot_base << ";\n";
+    os << "      default: return " << g.nslots << ";\n    }\n  }\n";
+    os << "  static DEV void cbody(int ci, Ctx<" << g.K << "> &c, const u32 (&pl)[8][" << g.K
+       << "], const u32 *st, u32 *nst, const u32 rmask) {\n    (void)ci; (void)c; (void)pl; (void)st; (void)nst; (void)rmask;\n";
+    if (gen_cm) {
+      os << "    switch (ci) {\n";
+      for (int ci = 0; ci < NC; ++ci) os << "      case " << ci << ": cb" << ci << "(c, pl, st, nst, rmask); break;\n";
+      os << "      default: break;\n    }\n";
     }
     os << "  }\n};\n";
     const int LB = lit_scratch_bytes(cs);
@@ -629,7 +663,20 @@ std::string emit_kernel_unit(CompiledSet &cs) {
         "  const int cpg = (p.nseg_max + wpb - 1) / wpb;  // CTAs per group\n"
         "  const int g = (int)(blockIdx.x / cpg);\n"
         "  const long long seg = (long long)(blockIdx.x % cpg) * wpb + warp;\n"
-        "  if (g >= RX_NG) return;\n"
+        "  if (p.task_ctr) {\n"
+        "    // dynamic: every warp pulls (group, segment) tasks, group-major, from\n"
+        "    // one counter until they run out (load balance under zero skipping)\n"
+        "    const long long ntask = (long long)RX_NG * p.nseg_max;\n"
+        "    for (;;) {\n"
+        "      unsigned long long t = 0;\n"
+        "      if ((threadIdx.x & 31) == 0) t = atomicAdd(p.task_ctr, 1ull);\n"
+        "      t = __shfl_sync(RX_FULL, t, 0);\n"
+        "      if ((long long)t >= ntask) return;\n"
+        "      const int tg = (int)(t / p.nseg_max), ts = (int)(t % p.nseg_max);\n"
+        "      switch (tg) {\n";
+  for (int gi = 0; gi < G; ++gi) os << "        case " << gi << ": rx_seg_" << gi << "(p, ts); break;\n";
+  os << "        default: break;\n      }\n      __syncwarp();\n    }\n  }\n";
+  os << "  if (g >= RX_NG) return;\n"
         "  switch (g) {\n";
   for (int gi = 0; gi < G; ++gi) os << "    case " << gi << ": rx_seg_" << gi << "(p, (int)seg); break;\n";
   os << "    default: break;\n  }\n}\n";

@@ -314,6 +314,9 @@ struct RxParams {
   int fix_phase;            // mode 1: 0 = serial fix-up, 1 = parallel per segment, 2 = serial remainder
   u32 *seg_fix;             // [nseg_max][G][NSMAX]: phase-1 end state of a segment that did not converge
   u32 *seg_nc;              // [nseg_max][G]: that segment did not converge in phase 1
+  u64 *task_ctr;            // pass 1: non-null = persistent warps pull (group, segment) tasks from it
+  int cmajor;               // sparse pass 1 runs cluster by cluster (rx_run_segment_cm)
+  int cm_sync;              // ... with one CTA barrier per cluster (static task map only)
 };
 
 template <int K> DEV void rx_load_window(const RxParams &p, Ctx<K> &c, u32 (&pl)[8][K], i64 fword) {
@@ -538,6 +541,9 @@ template <class G> DEV void rx_run_segment_pf(const RxParams &p, int seg, u64 *a
 template <class G>
 DEV void rx_run_segment_pf_staged(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *tbuf, u64 *bar,
                                   unsigned char *lb);
+template <class G>
+DEV void rx_run_segment_cm(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *tbuf, u64 *bar,
+                           unsigned char *lb);
 
 template <class G>
 DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *tbuf, u64 *bars,
@@ -546,7 +552,9 @@ DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned
   constexpr u32 WB = 1024u * K;  // window bytes
   if constexpr (G::PF) {
     (void)WB;
-    if (K <= 4 && !p.lockstep && !p.dbg) rx_run_segment_pf_staged<G>(p, seg, acc, sst, tbuf, bars, lb);
+    if (K <= 4 && !p.lockstep && !p.dbg && p.cmajor && G::NC > 0)
+      rx_run_segment_cm<G>(p, seg, acc, sst, tbuf, bars, lb);
+    else if (K <= 4 && !p.lockstep && !p.dbg) rx_run_segment_pf_staged<G>(p, seg, acc, sst, tbuf, bars, lb);
     else rx_run_segment_pf<G>(p, seg, acc, sst, lb);
     return;
   }
@@ -1233,5 +1241,160 @@ DEV void rx_run_segment_pf_staged(const RxParams &p, int seg, u64 *acc, u32 *sst
     if (p.st_out && w_end == nwin)
       for (int s = (int)c.lane; s < NS; s += 32) p.st_out[G::SBASE + s] = st[s];
   }
+  rx_flush<G>(p, c);
+}
+
+// Cluster-major sparse pass 1 (the default).  The
+// segment is walked once per factor cluster of the group, running only that
+// cluster's out-of-line code (G::cbody) in the windows whose frame holds one
+// of its factors or into which its own state flows.  A cluster's code stays
+// in the SM's instruction caches across consecutive windows (one straight-
+// line body per window over the whole group thrashed them: the top stall was
+// "no instruction"), at the price of re-loading and re-transposing a window
+// for each cluster that runs in it.  Clusters own disjoint state slots, so
+// running them one after the other over the segment computes exactly what
+// the window-major order computes.  With cm_sync the CTA's warps (same group,
+// consecutive segments) step from cluster to cluster together.
+template <class G>
+DEV void rx_run_segment_cm(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *tbuf, u64 *bar,
+                           unsigned char *lb) {
+  constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw;
+  constexpr u32 WB = 1024u * K;
+  const i64 len_words = rx_div_up(p.len, 32);
+  const i64 nwin = rx_div_up(len_words, Bw);
+  const i64 w_begin = (i64)seg * p.sw;
+  const bool live = w_begin < nwin || seg == 0;
+  const i64 w_end = !live ? w_begin : (w_begin + p.sw < nwin ? w_begin + p.sw : nwin);
+  Ctx<K> c;
+  rx_ctx_init<G>(p, c, acc, lb);
+  u32 pl[8][K];
+  u32 xr[K][8];
+  u32 *st = sst, *nst = sst + G::NSMAX;
+  if (c.lane == 0) rx_mbar_init(bar, 1);
+  __syncwarp();
+  const RxRange ir = rx_interior(p);
+  const u32 *gb = p.pf_gbits + (i64)G::GID * p.pf_ntiles;
+  const u32 *mm = p.pf_mmask + (i64)G::GID * 32 * p.pf_ntiles;
+  auto frame_blocks = [&](i64 w, i64 &b0, i64 &b1) {
+    i64 flo = (w * Bw - Lw) * 32, fhi = flo + 1024 * K;
+    if (flo < p.avail_lo) flo = p.avail_lo;
+    if (fhi > p.avail_hi) fhi = p.avail_hi;
+    if (fhi <= flo) fhi = flo + 1;
+    b0 = (flo - p.avail_lo) >> 10;
+    b1 = (fhi - 1 - p.avail_lo) >> 10;
+  };
+  i64 bmax = 0;
+  if (w_begin < w_end) {
+    i64 t0;
+    frame_blocks(w_end - 1, t0, bmax);
+  }
+  // members of the group whose factor occurs in window w's frame
+  auto frame_hits = [&](i64 w) -> u32 {
+    i64 b0, b1;
+    frame_blocks(w, b0, b1);
+    u32 mine = 0u;
+    for (i64 b = b0 + c.lane; b <= b1; b += 32)
+      if ((gb[b >> 5] >> (b & 31)) & 1u) mine |= mm[b];
+    return __reduce_or_sync(RX_FULL, mine);
+  };
+  // first window >= w whose frame holds a factor of the group (w_end if none)
+  auto next_group_hit = [&](i64 w) -> i64 {
+    if (w >= w_end) return w_end;
+    i64 b0, b1;
+    frame_blocks(w, b0, b1);
+    const i64 b = rx_pf_next(gb, b0, bmax, c.lane);
+    if (b > bmax) return w_end;
+    if (b <= b1) return w;
+    const i64 pos = p.avail_lo + b * RX_PF_BLK;
+    const i64 wn = rx_floor_div(rx_floor_div(pos, 32) + Lw - 32 * K, Bw) + 1;
+    const i64 r = wn > w + 1 ? wn : w + 1;
+    return r < w_end ? r : w_end;
+  };
+  i64 staged = -1;
+  u32 phase = 0;
+  auto stage = [&](i64 w) {
+    const i64 f = w * Bw - Lw;
+    if (w < w_end && f >= ir.lo && f + 32 * K <= ir.hi) {
+      __syncwarp();
+      if (c.lane == 0) rx_bulk_load(tbuf, p.in + f * 32, WB, bar);
+      staged = w;
+    }
+  };
+  auto retire = [&]() {
+    rx_mbar_wait(bar, phase);
+    phase ^= 1u;
+    staged = -1;
+  };
+  for (int ci = 0; ci < G::NC; ++ci) {
+    const int s0 = G::cslot(ci), s1 = G::cslot(ci + 1);
+    const u32 cm = G::cmask(ci);
+    const bool always = G::calways(ci);
+    for (int s = s0 + (int)c.lane; s < s1; s += 32) st[s] = (seg == 0 && p.st_in) ? p.st_in[G::SBASE + s] : 0u;
+    __syncwarp();
+    auto pending = [&](const u32 *a) -> bool {
+      bool any = false;
+      for (int s = s0 + (int)c.lane; s < s1; s += 32) any = any || a[s] != 0u;
+      return __any_sync(RX_FULL, any);
+    };
+    // first window >= w in which this cluster must run (no state pending)
+    auto next_c = [&](i64 w) -> i64 {
+      if (always) return w < w_end ? w : w_end;
+      for (;;) {
+        w = next_group_hit(w);
+        if (w >= w_end) return w_end;
+        if (frame_hits(w) & cm) return w;
+        ++w;
+      }
+    };
+    i64 w = pending(st) ? w_begin : next_c(w_begin);
+    if (w < w_end) stage(w);
+    while (w < w_end) {
+      const bool pend_in = pending(st);
+      const i64 fword = w * Bw - Lw;
+      if (staged == w) {
+        retire();
+        const uint4 *q = reinterpret_cast<const uint4 *>(tbuf + c.lane * (32u * K));
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+          const uint4 a0 = q[2 * k], a1 = q[2 * k + 1];
+          xr[k][0] = a0.x; xr[k][1] = a0.y; xr[k][2] = a0.z; xr[k][3] = a0.w;
+          xr[k][4] = a1.x; xr[k][5] = a1.y; xr[k][6] = a1.z; xr[k][7] = a1.w;
+        }
+      } else {
+        if (staged >= 0 && staged < w) retire();
+        rx_fetch<K>(p, ir, c.lane, xr, fword);
+      }
+      if (staged < 0) stage(pend_in ? w + 1 : next_c(w + 1));
+      const u32 rmask = frame_hits(w) & cm;
+      if (p.stats && c.lane == 0) {
+        atomicAdd(&p.stats[0], 1ull);
+        if (rmask == 0u) atomicAdd(&p.stats[1], 1ull);
+        atomicAdd(&p.stats[2], (u64)__popc(rmask));
+        atomicAdd(&p.stats[3], 1ull);
+      }
+      c.cw = (u32)((len_words - w * Bw) < Bw ? (len_words - w * Bw) : Bw);
+      c.word0 = fword;
+      rx_unpack<K>(p, ir, c, xr, pl, fword);
+      rx_commit_mask(p, ir, c, Lw, fword);
+      for (int s = s0 + (int)c.lane; s < s1; s += 32) nst[s] = 0u;
+      __syncwarp();
+      G::cbody(ci, c, pl, st, nst, rmask);
+      u32 *t = st;
+      st = nst;
+      nst = t;
+      __syncwarp();
+      w = pending(st) ? w + 1 : next_c(w + 1);
+    }
+    if (staged >= 0) retire();
+    if (live && s1 > s0) {
+      u32 *dst = p.seg_state + ((i64)seg * G::NG + G::GID) * G::NSMAX;
+      for (int s = s0 + (int)c.lane; s < s1; s += 32) dst[s] = st[s];
+      if (p.st_out && w_end == nwin)
+        for (int s = s0 + (int)c.lane; s < s1; s += 32) p.st_out[G::SBASE + s] = st[s];
+    }
+    __syncwarp();
+    if (p.cm_sync) __syncthreads();
+  }
+  if (!live) return;
   rx_flush<G>(p, c);
 }

@@ -498,6 +498,9 @@ struct RxParamsHost {  // must mirror RxParams in rx_device.cuh
   int fix_phase;
   unsigned int *seg_fix;
   unsigned int *seg_nc;
+  unsigned long long *task_ctr;
+  int cmajor;
+  int cm_sync;
 };
 
 rx_status ensure_loaded(rx_program *p, int &device) {
@@ -662,8 +665,23 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
   // segments: enough warps to fill the GPU several times over
   long long max_nwin = 0;
   for (auto &g : p->cs.groups) max_nwin = std::max(max_nwin, div_up(len_words, g.Bw));
-  // pass-1 CTAs: 16 segments of one group each; aim for ~4 waves of 148 SMs
-  const long long target_ctas = 148LL * 4;
+  // pass-1 CTAs: 16 segments of one group each; aim for ~4 waves of 148 SMs.
+  // Dynamic (sparse) mode: ~16 (group, segment) tasks per resident warp so
+  // that the dynamic queue evens out the data-dependent work
+  // experiment knobs: RX_DYNAMIC=1 persistent
+  // warps pulling (group, segment) tasks; RX_CMAJOR=0 window-major sparse
+  // pass; RX_CM_SYNC=0 no CTA barrier between clusters
+  const char *pls = getenv("RX_PF_LOCKSTEP"), *dys = getenv("RX_DYNAMIC");
+  const bool dynamic = p->cs.use_pf && !(pls && *pls == '1') && (dys && *dys == '1');
+  {
+    const char *e1 = getenv("RX_CMAJOR"), *e2 = getenv("RX_CM_SYNC");
+    prm.cmajor = (e1 && *e1 == '0') ? 0 : 1;
+    prm.cm_sync = (e2 && *e2 == '0') || dynamic ? 0 : 1;
+  }
+  long long waves = 16;  // RX_WAVES: pass-1 CTA waves per SM (measured best for the Snort-like set; knob)
+  if (const char *e = getenv("RX_WAVES"))
+    if (atoi(e) > 0) waves = atoi(e);
+  const long long target_ctas = 148LL * waves;
   const long long cpg0 = std::max<long long>(1, div_up(target_ctas, std::max(G, 1)));
   long long sw = std::max<long long>(4, div_up(max_nwin, cpg0 * kPass1Warps));
   long long nseg_max = std::max<long long>(1, div_up(max_nwin, sw));
@@ -719,7 +737,21 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
       const char *de = getenv("RX_DBG");  // timing experiments only: results are wrong when set
       prm.dbg = (de && *de) ? atoi(de) : 0;
     }
-    s = launch(p, m, m.pass1, cpg * mg, kPass1Warps, prm, stream);
+    // sparse (prefilter, no lockstep): a persistent grid pulling (group,
+    // segment) tasks dynamically; otherwise the static group-per-CTA map
+    long long p1_blocks = cpg * mg;
+    void *tctr = nullptr;
+    {
+      if (dynamic && prm.pf_on && !prm.lockstep) {
+        if (cudaMallocAsync(&tctr, 8, stream) != cudaSuccess) return fail(RX_ENOMEM, "task counter");
+        cudaMemsetAsync(tctr, 0, 8, stream);
+        prm.task_ctr = (unsigned long long *)tctr;
+        p1_blocks = std::min<long long>(p1_blocks, 148LL);
+      }
+    }
+    s = launch(p, m, m.pass1, p1_blocks, kPass1Warps, prm, stream);
+    prm.task_ctr = nullptr;
+    if (tctr) cudaFreeAsync(tctr, stream);
     prm.stats = nullptr;
     if (stats) {
       unsigned long long h[8];
