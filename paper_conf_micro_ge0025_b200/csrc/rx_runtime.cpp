@@ -7,6 +7,7 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <nvrtc.h>
+#include <zlib.h>
 
 #include <algorithm>
 #include <atomic>
@@ -117,6 +118,31 @@ bool read_file(const std::string &path, std::string &out) {
   return !out.empty();
 }
 
+// gzip-compressed cache entries (cubins compress ~5x; the in-tree cache
+// travels to the GPU box with the repo snapshot)
+bool read_gz(const std::string &path, std::string &out) {
+  gzFile f = gzopen(path.c_str(), "rb");
+  if (!f) return false;
+  out.clear();
+  char buf[1 << 16];
+  int n;
+  while ((n = gzread(f, buf, sizeof buf)) > 0) out.append(buf, (size_t)n);
+  const bool ok = n == 0;
+  gzclose(f);
+  return ok && !out.empty();
+}
+
+void write_gz_atomic(const std::string &path, const std::string &data) {
+  std::string tmp = path + ".tmp" + std::to_string(getpid()) + "_" +
+                    std::to_string((unsigned long long)std::hash<std::thread::id>{}(std::this_thread::get_id()));
+  gzFile f = gzopen(tmp.c_str(), "wb6");
+  if (!f) return;
+  const bool ok = gzwrite(f, data.data(), (unsigned)data.size()) == (int)data.size();
+  gzclose(f);
+  if (ok) rename(tmp.c_str(), path.c_str());
+  else unlink(tmp.c_str());
+}
+
 void write_file_atomic(const std::string &path, const std::string &data) {
   std::string tmp = path + ".tmp" + std::to_string(getpid()) + "_" +
                     std::to_string(std::hash<std::thread::id>()(std::this_thread::get_id()));
@@ -144,7 +170,7 @@ bool nvrtc_compile(const std::string &src, int max_regs, bool use_cache, std::st
   snprintf(hex, sizeof hex, "%016llx", (unsigned long long)fnv1a(key_src));
   std::string dir = cache_dir();
   std::string path = dir + "/" + hex + ".cubin";
-  if (use_cache && read_file(path, cubin)) return true;
+  if (use_cache && (read_gz(path + ".gz", cubin) || read_file(path, cubin))) return true;
   nvrtcProgram prog;
   if (nvrtcCreateProgram(&prog, src.c_str(), "rx_program.cu", 0, nullptr, nullptr) != NVRTC_SUCCESS) {
     log = "nvrtcCreateProgram failed";
@@ -170,7 +196,7 @@ bool nvrtc_compile(const std::string &src, int max_regs, bool use_cache, std::st
   nvrtcDestroyProgram(&prog);
   if (use_cache) {
     mkdirs(dir);
-    write_file_atomic(path, cubin);
+    write_gz_atomic(path + ".gz", cubin);
   }
   return true;
 }
