@@ -284,7 +284,7 @@ struct RegexEmitter {
         std::string t = fresh();
         os << I << "V<" << K << "> " << t << "i;\n";
         for (int i = 0; i < K; ++i) os << I << t << "i.w[" << i << "] = " << W(A, i) << ";\n";
-        os << I << "const V<" << K << "> " << t << "o = rx_lit<" << K << ">(c, " << t << "i, " << lit_pool << " + "
+        os << I << "const V<" << K << "> " << t << "o = rx_lit<" << K << ">(c.lane, c.wb, c.ob, " << t << "i, " << lit_pool << " + "
            << lit_off[n.cc] << ", " << n.k << ");\n";
         decl(in, nv(id), [&](int i) { return t + "o.w[" + std::to_string(i) + "]"; });
         break;
@@ -546,8 +546,9 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
     std::vector<uint32_t> cmask(NC, 0u);
     for (int ci = 0; ci < NC; ++ci)
       for (int m : g.clusters[ci].members) cmask[ci] |= 1u << m;
-    auto emit_fn = [&](const std::string &name, int c0, int c1) {
-      os << "  static __device__ __noinline__ void " << name << "(Ctx<" << g.K << "> &c, const u32 (&pl)[8][" << g.K
+    auto emit_fn = [&](const std::string &name, int c0, int c1, bool inl = false) {
+      os << "  static __device__ " << (inl ? "__forceinline__" : "__noinline__") << " void " << name << "(Ctx<" << g.K
+         << "> &c, const u32 (&pl)[8][" << g.K
          << "], const u32 *st, u32 *nst, const u32 rmask) {\n";
       os << "    (void)st; (void)nst; (void)rmask;\n";
       os << "    const u32 lane = c.lane; const int cw = (int)c.cw; (void)cw; (void)lane;\n";
@@ -590,6 +591,10 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
       os << "  }\n";
     };
     emit_fn("body", 0, NC);
+    // the same program inlined into pass 1's sparse runner: the basis planes
+    // and the window context stay in registers (the out-of-line call kept
+    // them in local memory, ~1.2 GB of DRAM writes per Snort-like step)
+    emit_fn("body_i", 0, NC, true);
     if (gen_cm)
       for (int ci = 0; ci < NC; ++ci) emit_fn("cb" + std::to_string(ci), ci, ci + 1);
     os << "  static constexpr int NC = " << (gen_cm ? NC : 0) << ";\n";

@@ -197,7 +197,8 @@ __device__ __noinline__ void rx_emit(const Ctx<K> c, int r, const V<K> v) {
 // (read as 0) never confirm.
 // ---------------------------------------------------------------------------
 template <int K>
-__device__ __noinline__ V<K> rx_lit(const Ctx<K> &c, const V<K> v, const unsigned char *lit, int n) {
+__device__ __noinline__ V<K> rx_lit(const u32 lane, const unsigned char *wb, u32 *ob, const V<K> v,
+                                    const unsigned char *lit, int n) {
   V<K> r;
   u32 any = 0u;
 #pragma unroll
@@ -207,11 +208,9 @@ __device__ __noinline__ V<K> rx_lit(const Ctx<K> &c, const V<K> v, const unsigne
     for (int i = 0; i < K; ++i) r.w[i] = 0u;
     return r;
   }
-  u32 *ob = c.ob;
 #pragma unroll
-  for (int i = 0; i < K; ++i) ob[c.lane * K + i] = 0u;
+  for (int i = 0; i < K; ++i) ob[lane * K + i] = 0u;
   __syncwarp();
-  const unsigned char *wb = c.wb;
   const int F = 1024 * K;
   const unsigned char l0 = lit[0];
 #pragma unroll
@@ -220,7 +219,7 @@ __device__ __noinline__ V<K> rx_lit(const Ctx<K> &c, const V<K> v, const unsigne
     while (b) {
       const int t = __ffs(b) - 1;
       b &= b - 1u;
-      const int q = (int)((c.lane * K + i) * 32u) + t;
+      const int q = (int)((lane * K + i) * 32u) + t;
       const int e = q + n;
       if (e >= F || wb[q + 1] != l0) continue;
       int j = 1;
@@ -230,7 +229,7 @@ __device__ __noinline__ V<K> rx_lit(const Ctx<K> &c, const V<K> v, const unsigne
   }
   __syncwarp();
 #pragma unroll
-  for (int i = 0; i < K; ++i) r.w[i] = ob[c.lane * K + i];
+  for (int i = 0; i < K; ++i) r.w[i] = ob[lane * K + i];
   __syncwarp();
   return r;
 }
@@ -1226,7 +1225,7 @@ DEV void rx_run_segment_pf_staged(const RxParams &p, int seg, u64 *acc, u32 *sst
     rx_unpack<K>(p, ir, c, xr, pl, fword);
     rx_commit_mask(p, ir, c, Lw, fword);
     if (NS > 0) rx_state_zero(nst, NS, c.lane);
-    G::body(c, pl, st, nst, rmask);
+    G::body_i(c, pl, st, nst, rmask);
     u32 *t = st;
     st = nst;
     nst = t;

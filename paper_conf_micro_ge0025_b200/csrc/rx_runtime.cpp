@@ -240,7 +240,28 @@ struct rx_program {
   std::vector<Ev> prof_ev;
   double prof_ms[3] = {0, 0, 0};
   uint64_t prof_n[3] = {0, 0, 0};
+  // device scratch per stream (grow-only, reused call after call): a
+  // cudaMallocAsync/cudaFreeAsync pair per buffer per call left the GPU idle
+  // between steps (7.5 ms per Snort-like step, 55 ms per Dotstar-like step)
+  std::map<std::pair<void *, int>, std::pair<void *, size_t>> scratch;
 };
+
+namespace {
+// scratch slots of one rx_match call
+enum { SC_STATUS = 0, SC_SEGSTATE = 1, SC_PF = 2, SC_TASK = 3, SC_FIX = 4 };
+void *scratch_get(rx_program *p, cudaStream_t s, int slot, size_t bytes) {
+  std::lock_guard<std::mutex> lk(p->mu);
+  auto &e = p->scratch[{(void *)s, slot}];
+  if (e.second < bytes) {
+    if (e.first) cudaFree(e.first);  // synchronising; growth only
+    e.first = nullptr;
+    e.second = 0;
+    if (cudaMalloc(&e.first, bytes) != cudaSuccess) return nullptr;
+    e.second = bytes;
+  }
+  return e.first;
+}
+}  // namespace
 
 extern "C" {
 
@@ -303,6 +324,8 @@ void rx_free(rx_program *p) {
       if (m.pf_mem) cudaFree(m.pf_mem);
       if (cur != m.device && cur >= 0) cudaSetDevice(cur);
     }
+  for (auto &kv : p->scratch)
+    if (kv.second.first) cudaFree(kv.second.first);
   delete p;
 }
 
@@ -669,7 +692,7 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
   (void)dummy_status_host;
   unsigned int *status_scratch = nullptr;
   if (!prm.status) {
-    if (cudaMallocAsync((void **)&status_scratch, 4, stream) != cudaSuccess) return fail(RX_ENOMEM, "status");
+    if (!(status_scratch = (unsigned int *)scratch_get(p, stream, SC_STATUS, 256))) return fail(RX_ENOMEM, "status");
     cudaMemsetAsync(status_scratch, 0, 4, stream);
     prm.status = status_scratch;
   }
@@ -685,7 +708,6 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
       s = launch(p, m, m.fixup, div_up(m.g_end - m.g_begin, kFixupWarps), kFixupWarps, prm, stream);
       if (s != RX_OK) return s;
     }
-    if (status_scratch) cudaFreeAsync(status_scratch, stream);
     return RX_OK;
   }
   // segments: enough warps to fill the GPU several times over
@@ -720,7 +742,7 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
     unsigned int *seg_state = nullptr;
     size_t bytes = 4ull * (size_t)nseg_max * (size_t)mg * (size_t)std::max(1, m.ns_max);
     if (m.any_state) {
-      if (cudaMallocAsync((void **)&seg_state, bytes, stream) != cudaSuccess) return fail(RX_ENOMEM, "seg_state");
+      if (!(seg_state = (unsigned int *)scratch_get(p, stream, SC_SEGSTATE, bytes))) return fail(RX_ENOMEM, "seg_state");
     }
     prm.seg_state = seg_state;
     prm.mode = 0;
@@ -730,7 +752,7 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
       const long long ntiles = std::max<long long>(1, div_up(span, 32768));
       const size_t gb_bytes = (size_t)4 * (size_t)ntiles * (size_t)mg;
       const size_t bl_bytes = (size_t)4 * 32 * (size_t)ntiles * (size_t)mg;
-      if (cudaMallocAsync(&pf_scratch, gb_bytes + bl_bytes + 256, stream) != cudaSuccess)
+      if (!(pf_scratch = scratch_get(p, stream, SC_PF, gb_bytes + bl_bytes + 256)))
         return fail(RX_ENOMEM, "prefilter scratch");
       prm.pf_tab = (const unsigned int *)m.pf_mem;
       prm.pf_words = (unsigned int)p->cs.pf.blob.size();
@@ -769,7 +791,7 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
     void *tctr = nullptr;
     {
       if (dynamic && prm.pf_on && !prm.lockstep) {
-        if (cudaMallocAsync(&tctr, 8, stream) != cudaSuccess) return fail(RX_ENOMEM, "task counter");
+        if (!(tctr = scratch_get(p, stream, SC_TASK, 256))) return fail(RX_ENOMEM, "task counter");
         cudaMemsetAsync(tctr, 0, 8, stream);
         prm.task_ctr = (unsigned long long *)tctr;
         p1_blocks = std::min<long long>(p1_blocks, 148LL);
@@ -777,7 +799,6 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
     }
     s = launch(p, m, m.pass1, p1_blocks, kPass1Warps, prm, stream);
     prm.task_ctr = nullptr;
-    if (tctr) cudaFreeAsync(tctr, stream);
     prm.stats = nullptr;
     if (stats) {
       unsigned long long h[8];
@@ -787,7 +808,6 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
               h[3], h[0], h[1], h[2]);
       cudaFree(stats);
     }
-    if (pf_scratch) cudaFreeAsync(pf_scratch, stream);
     prm.pf_on = 0;
     if (s != RX_OK) return s;
     if (m.any_state) {
@@ -801,7 +821,7 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
         // warp per group, only where a segment's carry outlived it
         void *fx = nullptr;
         const size_t nc_bytes = 4ull * (size_t)nseg_max * (size_t)mg;
-        if (cudaMallocAsync(&fx, bytes + nc_bytes + 256, stream) != cudaSuccess) return fail(RX_ENOMEM, "fix-up scratch");
+        if (!(fx = scratch_get(p, stream, SC_FIX, bytes + nc_bytes + 256))) return fail(RX_ENOMEM, "fix-up scratch");
         prm.seg_fix = (unsigned int *)fx;
         prm.seg_nc = (unsigned int *)((char *)fx + ((bytes + 255) & ~(size_t)255));
         cudaMemsetAsync(prm.seg_nc, 0, nc_bytes, stream);
@@ -812,13 +832,10 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
           s = launch(p, m, m.fixup, div_up(mg, kFixupWarps), kFixupWarps, prm, stream);
         }
         prm.fix_phase = 0;
-        cudaFreeAsync(fx, stream);
       }
       if (s != RX_OK) return s;
-      cudaFreeAsync(seg_state, stream);
     }
   }
-  if (status_scratch) cudaFreeAsync(status_scratch, stream);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(RX_ECUDA, cudaGetErrorString(e));
   return RX_OK;
