@@ -146,6 +146,23 @@ rx_status rx_rematch_chunk(const rx_program *p, const uint8_t *d_input, uint64_t
                            uint64_t halo_right, uint64_t global_offset, const void *d_state_assumed,
                            const void *d_state_true, void *d_state_out, void *stream, const rx_output *out);
 
+/* MIMD form ("a set of regular expressions ... over
+ * a shared input stream", extended to many independent streams, e.g. one per
+ * packet flow).  offsets: HOST u64[n_streams + 1], non-decreasing; stream i is
+ * d_input[offsets[i] .. offsets[i+1]) and is matched as a complete input of
+ * its own: zero state at its start, no byte of a neighbouring stream is ever
+ * read, so no match crosses a stream boundary.  Outputs are per stream:
+ * d_counts u64[n_streams][n_regex], d_digests u64[n_streams][n_regex][2]
+ * (stream-relative positions), d_bitstreams u32[n_streams][n_regex][pitch]
+ * (pitch_words >= ceil(max stream length / 32)); the match list is shared and
+ * holds positions relative to d_input (offsets[i] + i-th byte), so the stream
+ * of an entry is found by searching offsets.  All OVERWRITTEN.  Empty streams
+ * are valid.  Errors: RX_EINVAL for null pointers, decreasing offsets or a
+ * short pitch (nothing launched).  Asynchronous on `stream`; this first form
+ * issues one launch sequence per non-empty stream. */
+rx_status rx_match_batch(const rx_program *p, const uint8_t *d_input, const uint64_t *offsets, uint32_t n_streams,
+                         void *stream, const rx_output *out);
+
 /* Per-kernel device timing (for roofline reporting): when on, every launch
  * of the program is bracketed by CUDA events on its stream.  rx_kernel_times
  * waits for the recorded events and writes the accumulated milliseconds and

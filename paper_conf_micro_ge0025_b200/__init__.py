@@ -23,7 +23,7 @@ RX_F_NO_REBALANCE, RX_F_NO_GUARDS, RX_F_NO_CACHE, RX_F_REBALANCE, RX_F_NO_PREFIL
 
 EXPORTED = ["rx_compile", "rx_free", "rx_num_regex", "rx_num_groups", "rx_max_lookback", "rx_max_lookahead",
             "rx_boundary_bytes", "rx_program_source", "rx_program_info", "rx_match", "rx_match_chunk",
-            "rx_rematch_chunk", "rx_last_error", "rx_kernels_per_match", "rx_set_profiling", "rx_kernel_times"]
+            "rx_rematch_chunk", "rx_last_error", "rx_kernels_per_match", "rx_set_profiling", "rx_kernel_times", "rx_match_batch"]
 
 
 class RxError(RuntimeError):
@@ -80,6 +80,8 @@ def load_library():
         lib.rx_match_chunk.restype = ctypes.c_int
         lib.rx_rematch_chunk.argtypes = [vp, vp, u64, u64, u64, u64, vp, vp, vp, vp, ctypes.POINTER(_Output)]
         lib.rx_rematch_chunk.restype = ctypes.c_int
+        lib.rx_match_batch.argtypes = [vp, vp, vp, u32, vp, ctypes.POINTER(_Output)]
+        lib.rx_match_batch.restype = ctypes.c_int
         lib.rx_set_profiling.argtypes = [vp, ctypes.c_int]
         lib.rx_set_profiling.restype = ctypes.c_int
         lib.rx_kernel_times.argtypes = [vp, vp, vp, ctypes.c_int]
@@ -249,6 +251,37 @@ class Program:
                                           int(halo_right), int(global_offset), _ptr(state_assumed),
                                           _ptr(state_true), _ptr(state_out), _stream_handle(stream),
                                           ctypes.byref(s)))
+        return out
+
+    def match_batch(self, data, offsets, dense=False, digests=True, match_cap=None, stream=None):
+        """rx_match_batch: `data` a CUDA uint8 tensor holding the streams back
+        to back, `offsets` n_streams + 1 host ints.  Returns counts
+        int64[n_streams, n_regex], digests int64[n_streams, n_regex, 2],
+        dense int32[n_streams, n_regex, pitch]; match-list positions are
+        relative to `data`."""
+        import numpy as np
+        import torch
+        offs = np.ascontiguousarray(np.asarray(offsets, dtype=np.uint64))
+        ns = max(len(offs) - 1, 0)
+        n, dev = self.n_regex, data.device
+        max_len = int((offs[1:] - offs[:-1]).max()) if ns else 0
+        out = {"counts": torch.zeros((max(ns, 1), max(n, 1)), dtype=torch.int64, device=dev)[:ns, :n],
+               "digests": torch.zeros((max(ns, 1), max(n, 1), 2), dtype=torch.int64, device=dev)[:ns, :n]
+               if digests else None,
+               "status": torch.zeros(1, dtype=torch.int32, device=dev)}
+        if match_cap is not None:
+            out["matches"] = torch.zeros((max(int(match_cap), 1), 2), dtype=torch.int64, device=dev)
+            out["match_cap"] = int(match_cap)
+            out["match_total"] = torch.zeros(1, dtype=torch.int64, device=dev)
+        if dense:
+            pitch = max((max_len + 31) // 32, 1)
+            out["dense"] = torch.zeros((max(ns, 1), max(n, 1), pitch), dtype=torch.int32, device=dev)[:ns, :n]
+            out["pitch"] = pitch
+        else:
+            out["dense"], out["pitch"] = None, 0
+        s = self._out_struct(out)
+        _check(self._lib.rx_match_batch(self._h, _ptr(data), offs.ctypes.data_as(ctypes.c_void_p), ns,
+                                        _stream_handle(stream), ctypes.byref(s)))
         return out
 
     def set_profiling(self, on: bool = True):

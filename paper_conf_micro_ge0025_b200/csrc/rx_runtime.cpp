@@ -864,4 +864,45 @@ rx_status rx_rematch_chunk(const rx_program *p, const uint8_t *d_input, uint64_t
              d_state_out, d_state_assumed, 1, 2, (cudaStream_t)stream, out);
 }
 
+
+// SURVEY 8(f) N3 / P:L178 (MIMD: many independent input streams).  Stream i
+// is d_input[offsets[i] .. offsets[i+1]) and is matched as a whole input of
+// its own (zero state at its start, nothing readable past either end), so
+// no match and no state crosses a stream boundary.  This first form issues
+// one rx_match_chunk sequence per stream on `stream`; outputs are per stream.
+rx_status rx_match_batch(const rx_program *p, const uint8_t *d_input, const uint64_t *offsets, uint32_t n_streams,
+                         void *stream, const rx_output *out) {
+  if (!p || !out || !out->d_counts || (n_streams && !offsets)) return fail(RX_EINVAL, "null argument");
+  uint64_t max_len = 0;
+  for (uint32_t i = 0; i < n_streams; i++) {
+    if (offsets[i + 1] < offsets[i]) return fail(RX_EINVAL, "offsets must be non-decreasing");
+    max_len = std::max<uint64_t>(max_len, offsets[i + 1] - offsets[i]);
+  }
+  if (out->d_bitstreams && out->pitch_words < (max_len + 31) / 32) return fail(RX_EINVAL, "pitch_words too small");
+  cudaStream_t st = (cudaStream_t)stream;
+  const uint64_t n = p->n_regex;
+  const uint64_t ns = n_streams;
+  if (n && ns && cudaMemsetAsync(out->d_counts, 0, 8ull * n * ns, st) != cudaSuccess) return fail(RX_ECUDA, "memset");
+  if (n && ns && out->d_digests && cudaMemsetAsync(out->d_digests, 0, 16ull * n * ns, st) != cudaSuccess)
+    return fail(RX_ECUDA, "memset");
+  if (n && ns && out->d_bitstreams &&
+      cudaMemsetAsync(out->d_bitstreams, 0, 4ull * n * ns * out->pitch_words, st) != cudaSuccess)
+    return fail(RX_ECUDA, "memset");
+  if (out->d_status && cudaMemsetAsync(out->d_status, 0, 4, st) != cudaSuccess) return fail(RX_ECUDA, "memset");
+  if (out->d_match_total && cudaMemsetAsync(out->d_match_total, 0, 8, st) != cudaSuccess)
+    return fail(RX_ECUDA, "memset");
+  for (uint32_t i = 0; i < n_streams; i++) {
+    rx_output o = *out;
+    o.d_counts = out->d_counts + (uint64_t)i * n;
+    if (out->d_digests) o.d_digests = out->d_digests + 2ull * i * n;
+    if (out->d_bitstreams) o.d_bitstreams = out->d_bitstreams + (uint64_t)i * n * out->pitch_words;
+    const uint64_t len = offsets[i + 1] - offsets[i];
+    if (!len) continue;  // an empty stream has no matches (its slots are zeroed above)
+    rx_status s = run(const_cast<rx_program *>(p), d_input + offsets[i], len, 0, 0, offsets[i], nullptr, nullptr,
+                      nullptr, 1, 0, st, &o);
+    if (s != RX_OK) return s;
+  }
+  return RX_OK;
+}
+
 }  // extern "C"

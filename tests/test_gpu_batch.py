@@ -1,0 +1,80 @@
+"""GPU parity of rx_match_batch: many independent
+streams in one call.  Each stream must equal the oracle run on that stream
+alone -- bit-exact counts, digests and dense match-end bits -- so no match or
+carried state (MatchStar runs, while-loop frontiers) crosses a boundary.
+Streams are ragged, include empty ones, and are cut inside long matches."""
+import numpy as np
+import pytest
+
+import gen
+import oracle
+
+torch = pytest.importorskip("torch")
+rx = pytest.importorskip("paper_conf_micro_ge0025_b200")
+
+pytestmark = pytest.mark.gpu
+
+PATS = gen.tiny_patterns() + [rb"abcd.*xyz", rb"q[^z]*z", rb"(ab|cd)+e", rb"a[a-z]*b"]
+
+
+def _check_batch(pats, streams, offset_pad=0):
+    prog = rx.Program(pats)
+    data = b"".join(streams)
+    offs = np.cumsum([0] + [len(s) for s in streams]).astype(np.uint64)
+    buf = torch.zeros(len(data) + 64, dtype=torch.uint8, device="cuda")
+    if data:
+        buf[: len(data)] = torch.frombuffer(bytearray(data), dtype=torch.uint8).cuda()
+    cap = 1 << 16
+    out = prog.match_batch(buf[: len(data)], offs, dense=True, match_cap=cap)
+    torch.cuda.synchronize()
+    assert int(out["status"].cpu()[0]) == 0
+    counts = out["counts"].cpu().numpy().view(np.uint64)
+    digests = out["digests"].cpu().numpy().view(np.uint64)
+    dense = out["dense"].cpu().numpy().view(np.uint32)
+    reg, pos = rx.Program.match_list(out)
+    total = 0
+    for i, s in enumerate(streams):
+        o = oracle.run_set(pats, s, dense=True)
+        assert np.array_equal(counts[i], o["counts"]), (i, len(s))
+        assert np.array_equal(digests[i], o["digests"]), (i, len(s))
+        w = (len(s) + 31) // 32
+        for r in range(len(pats)):
+            assert np.array_equal(dense[i, r, :w], o["dense"][r][:w]), (i, pats[r])
+            assert not dense[i, r, w:].any()
+            # list entries of this stream are exactly the oracle's ends + offset
+            sel = (reg == r) & (pos >= offs[i]) & (pos < offs[i + 1])
+            bits = np.unpackbits(o["dense"][r][:w].view(np.uint8), bitorder="little")[: len(s)]
+            assert np.array_equal(pos[sel] - offs[i], np.nonzero(bits)[0].astype(np.uint64))
+        total += int(o["counts"].sum())
+    assert len(reg) == total
+
+
+def test_batch_ragged_streams_match_oracle_per_stream():
+    rng = np.random.default_rng(11)
+    base = gen.tiny_input()
+    cuts = sorted(set(int(x) for x in rng.integers(0, len(base), 23)) | {0, 5, 5, 37, 1024, 1025, len(base)})
+    streams = [base[a:b] for a, b in zip(cuts[:-1], cuts[1:])] + [b"", b"abc", b"a" + b"bc" * 3000 + b"d"]
+    _check_batch(PATS, streams)
+
+
+def test_batch_state_does_not_cross_boundaries():
+    # every match here would need bytes of two streams: none may be reported
+    streams = [b"ab", b"c", b"a" + b"bc" * 700, b"d", b"abcd", b"xyz", b"q" + b"y" * 5000, b"z", b"fo", b"o"]
+    _check_batch(PATS, streams)
+
+
+def test_batch_empty():
+    prog = rx.Program(PATS)
+    buf = torch.zeros(16, dtype=torch.uint8, device="cuda")
+    out = prog.match_batch(buf[:0], [0])
+    assert out["counts"].shape == (0, len(PATS))
+    out = prog.match_batch(buf[:0], [0, 0, 0])
+    torch.cuda.synchronize()
+    assert int(out["counts"].abs().sum()) == 0
+
+
+def test_batch_rejects_decreasing_offsets():
+    prog = rx.Program(PATS)
+    buf = torch.zeros(64, dtype=torch.uint8, device="cuda")
+    with pytest.raises(rx.RxError):
+        prog.match_batch(buf, [0, 40, 30, 64])
