@@ -94,3 +94,19 @@ def test_kernel_param_struct_mirrors_match():
     host = open(os.path.join(ROOT, "paper_conf_micro_ge0025_b200", "csrc", "rx_runtime.cpp")).read()
     a, b = _struct_fields(dev, "RxParams"), _struct_fields(host, "RxParamsHost")
     assert a == b, (a, b)
+
+
+def test_match_batch_validates_offsets_before_any_launch():
+    # host-side argument checks of rx_match_batch (include/rx.h) run before
+    # any CUDA call, so the C entry point is testable without a GPU
+    import ctypes
+    import numpy as np
+    p = rx.Program(gen.tiny_patterns())
+    counts = np.zeros(3 * p.n_regex, dtype=np.uint64)
+    o = rx._Output()
+    o.d_counts = counts.ctypes.data
+    bad = np.array([0, 40, 30, 64], dtype=np.uint64)
+    st = p._lib.rx_match_batch(p._h, None, bad.ctypes.data_as(ctypes.c_void_p), 3, None, ctypes.byref(o))
+    assert st == rx.RX_EINVAL and b"non-decreasing" in p._lib.rx_last_error()
+    st = p._lib.rx_match_batch(p._h, None, None, 3, None, ctypes.byref(o))
+    assert st == rx.RX_EINVAL
