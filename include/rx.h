@@ -128,8 +128,9 @@ typedef struct {
 rx_status rx_match(const rx_program *p, const uint8_t *d_input, uint64_t len, void *stream, const rx_output *out);
 
 /* Chunked / multi-GPU form: commit positions [0, len) of a chunk whose bytes
- * are readable at d_input[-halo_left .. len + halo_right).  Positions are
- * reported as global_offset + i (digests, bitstreams stay chunk-relative).
+ * are readable at d_input[-halo_left .. len + halo_right).  Positions in the
+ * match list and the digests are global_offset + i (so digests of chunks add
+ * up to the whole stream's); bitstreams stay chunk-relative.
  * d_state_in: nullable device blob of rx_boundary_bytes() (NULL = the chunk
  * starts the stream: zero state); d_state_out: nullable, receives the state
  * at the chunk end.  Counts/digests are ACCUMULATED when `accumulate` != 0. */
@@ -153,9 +154,9 @@ rx_status rx_rematch_chunk(const rx_program *p, const uint8_t *d_input, uint64_t
  * its own: zero state at its start, no byte of a neighbouring stream is ever
  * read, so no match crosses a stream boundary.  Outputs are per stream:
  * d_counts u64[n_streams][n_regex], d_digests u64[n_streams][n_regex][2]
- * (stream-relative positions), d_bitstreams u32[n_streams][n_regex][pitch]
- * (pitch_words >= ceil(max stream length / 32)); the match list is shared and
- * holds positions relative to d_input (offsets[i] + i-th byte), so the stream
+ * (over positions relative to d_input, like the match list), d_bitstreams u32[n_streams][n_regex][pitch]
+ * (pitch_words >= ceil(max stream length / 32); stream-relative bits); the
+ * match list is shared and holds positions relative to d_input (offsets[i] + i-th byte), so the stream
  * of an entry is found by searching offsets.  All OVERWRITTEN.  Empty streams
  * are valid.  Errors: RX_EINVAL for null pointers, decreasing offsets or a
  * short pitch (nothing launched).  Asynchronous on `stream`; this first form

@@ -256,7 +256,8 @@ class Program:
     def match_batch(self, data, offsets, dense=False, digests=True, match_cap=None, stream=None):
         """rx_match_batch: `data` a CUDA uint8 tensor holding the streams back
         to back, `offsets` n_streams + 1 host ints.  Returns counts
-        int64[n_streams, n_regex], digests int64[n_streams, n_regex, 2],
+        int64[n_streams, n_regex], digests int64[n_streams, n_regex, 2] (over
+        positions relative to `data`),
         dense int32[n_streams, n_regex, pitch]; match-list positions are
         relative to `data`."""
         import numpy as np
@@ -265,7 +266,8 @@ class Program:
         ns = max(len(offs) - 1, 0)
         n, dev = self.n_regex, data.device
         max_len = int((offs[1:] - offs[:-1]).max()) if ns else 0
-        out = {"counts": torch.zeros((max(ns, 1), max(n, 1)), dtype=torch.int64, device=dev)[:ns, :n],
+        counts_full = torch.zeros((max(ns, 1), max(n, 1)), dtype=torch.int64, device=dev)
+        out = {"counts": counts_full[:ns, :n],
                "digests": torch.zeros((max(ns, 1), max(n, 1), 2), dtype=torch.int64, device=dev)[:ns, :n]
                if digests else None,
                "status": torch.zeros(1, dtype=torch.int32, device=dev)}
@@ -280,6 +282,7 @@ class Program:
         else:
             out["dense"], out["pitch"] = None, 0
         s = self._out_struct(out)
+        s.d_counts = counts_full.data_ptr()  # an empty view may report a null pointer
         _check(self._lib.rx_match_batch(self._h, _ptr(data), offs.ctypes.data_as(ctypes.c_void_p), ns,
                                         _stream_handle(stream), ctypes.byref(s)))
         return out

@@ -16,7 +16,7 @@ with open(det, newline="") as f:
 hdr = next(r for r in rows if "Metric Name" in r)
 ix = {c: i for i, c in enumerate(hdr)}
 for r in rows[rows.index(hdr) + 1:]:
-    if len(r) != len(hdr):
+    if len(r) <= ix["Metric Value"]:
         continue
     k = (r[ix["ID"]], r[ix["Kernel Name"]].split("(")[0])
     d = launches.setdefault(k, {})
