@@ -225,6 +225,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--length-mib", type=int, default=0, help="input bytes per GPU (default: the config's)")
     ap.add_argument("--no-prefilter", action="store_true", help="ablation: RX_F_NO_PREFILTER")
+    ap.add_argument("--words-per-lane", type=int, default=0, help="experiment: minimum K (rx_options.words_per_lane)")
+    ap.add_argument("--group-size", type=int, default=0, help="experiment: max regexes per group (rx_options)")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -244,7 +246,8 @@ def main():
     pats, data, nbytes, name = load_workload(args.config, (args.length_mib << 20) if args.length_mib else None, rank)
     nbytes = int(data.size)
     t0 = time.perf_counter()
-    prog = rx.Program(pats, flags=rx.RX_F_NO_PREFILTER if args.no_prefilter else 0)
+    prog = rx.Program(pats, flags=rx.RX_F_NO_PREFILTER if args.no_prefilter else 0,
+                      words_per_lane=args.words_per_lane or None, group_size=args.group_size or None)
     compile_s = time.perf_counter() - t0
 
     host = torch.from_numpy(np.ascontiguousarray(data)).pin_memory()
@@ -335,7 +338,9 @@ def main():
                    "groups": prog.n_groups, "outputs": "per-regex counts (dense streams off: 31 GiB at this size)",
                    "l2": f"input {nbytes >> 20} MiB per GPU" + (" > 126 MB L2: no flush needed" if nbytes > (126 << 20)
                                                                   else " < L2: L2 flushed between steps"),
-                   "prefilter": not args.no_prefilter, "compile_s": round(compile_s, 1)},
+                   "prefilter": not args.no_prefilter, "compile_s": round(compile_s, 1),
+                   **({"words_per_lane": args.words_per_lane} if args.words_per_lane else {}),
+                   **({"group_size": args.group_size} if args.group_size else {})},
         "roofline": roofline(ktimes, nbytes, len(pats), hbm, hbm_src, name, ms),
         "clocks": clocks,
         "gpu_launches": sum(v[1] for v in ktimes.values()) or launches_per_step * args.steps,
