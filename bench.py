@@ -97,6 +97,14 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(self.rows)}
 
 
+# Per-workload compile options of the timed launch configuration (the GPU
+# parity tests build the same program: tests/test_gpu_fullsize.py,
+# tests/test_gpu_configs.py).  Snort-like: K = 4 words per lane (4096
+# positions per warp window) measured 24.4 vs 20.2 GB/s at K = 2; the
+# Dotstar-like set is slower at K = 4 (4.1 vs 5.2 GB/s: coarser skipping), so
+# the others keep the compiler's default.
+PROGRAM_OPTS = {"snort": {"words_per_lane": 4}}
+
 WORKLOADS = {
     # name: (pattern builder, input builder(length, rank), default bytes per GPU, description)
     "snort": (lambda: __import__("gen").snort_patterns(1000, 2)[0],
@@ -246,8 +254,12 @@ def main():
     pats, data, nbytes, name = load_workload(args.config, (args.length_mib << 20) if args.length_mib else None, rank)
     nbytes = int(data.size)
     t0 = time.perf_counter()
-    prog = rx.Program(pats, flags=rx.RX_F_NO_PREFILTER if args.no_prefilter else 0,
-                      words_per_lane=args.words_per_lane or None, group_size=args.group_size or None)
+    popts = dict(PROGRAM_OPTS.get(args.config, {}))
+    if args.words_per_lane:
+        popts["words_per_lane"] = args.words_per_lane
+    if args.group_size:
+        popts["group_size"] = args.group_size
+    prog = rx.Program(pats, flags=rx.RX_F_NO_PREFILTER if args.no_prefilter else 0, **popts)
     compile_s = time.perf_counter() - t0
 
     host = torch.from_numpy(np.ascontiguousarray(data)).pin_memory()
@@ -339,8 +351,7 @@ def main():
                    "l2": f"input {nbytes >> 20} MiB per GPU" + (" > 126 MB L2: no flush needed" if nbytes > (126 << 20)
                                                                   else " < L2: L2 flushed between steps"),
                    "prefilter": not args.no_prefilter, "compile_s": round(compile_s, 1),
-                   **({"words_per_lane": args.words_per_lane} if args.words_per_lane else {}),
-                   **({"group_size": args.group_size} if args.group_size else {})},
+                   **popts},
         "roofline": roofline(ktimes, nbytes, len(pats), hbm, hbm_src, name, ms),
         "clocks": clocks,
         "gpu_launches": sum(v[1] for v in ktimes.values()) or launches_per_step * args.steps,

@@ -27,8 +27,8 @@ def _run(prog, data: np.ndarray):
             int(out["status"].cpu()[0]))
 
 
-def _parity(pats, data, min_total=1):
-    prog = rx.Program(pats)
+def _parity(pats, data, min_total=1, **opts):
+    prog = rx.Program(pats, **opts)
     counts, digests, status = _run(prog, data)
     o = oracle.run_set(pats, bytes(data))
     assert status == 0
@@ -43,6 +43,12 @@ def _parity(pats, data, min_total=1):
 def test_config2_snort_like_prefix():
     pats = gen.snort_patterns(1000, 2)[0]
     _parity(pats, gen.snort_input((4 << 20) + 12345, seed=2))
+
+
+def test_config2_snort_like_prefix_bench_k4():
+    # the bench's compile options for this workload (bench.PROGRAM_OPTS: K = 4)
+    pats = gen.snort_patterns(1000, 2)[0]
+    _parity(pats, gen.snort_input((4 << 20) + 12345, seed=2), words_per_lane=4)
 
 
 def test_config3_clamav_brill_prefix():

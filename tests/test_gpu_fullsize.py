@@ -48,7 +48,7 @@ def _splitmix64(x: np.ndarray) -> np.ndarray:
 
 def _full_run(config, cap):
     pats, data, nbytes, _ = bench.load_workload(config)
-    prog = rx.Program(pats)
+    prog = rx.Program(pats, **bench.PROGRAM_OPTS.get(config, {}))  # the bench's launch configuration
     dev = torch.device("cuda", 0)
     d_in = torch.from_numpy(np.ascontiguousarray(data)).to(dev)
     out = prog.alloc_outputs(nbytes, dev, dense=False, digests=True, match_cap=cap)
