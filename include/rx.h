@@ -63,7 +63,8 @@ typedef struct {
   uint32_t interval;       /* zero-block-skipping guard interval in IR instructions (Sec. 6); 0 = default 8; UINT32_MAX = no guards */
   uint32_t max_regs;       /* NVRTC --maxrregcount; 0 = default 128 */
   uint32_t group_size;     /* max regexes per group; 0 = auto */
-  uint32_t words_per_lane; /* K: 32-bit words per lane per window (window = 1024*K positions); 0 = auto */
+  uint32_t words_per_lane; /* K: 32-bit words per lane per window (window = 1024*K positions): 0 (auto), 1, 2, 4
+                              or 8; anything else is RX_EINVAL */
   uint32_t flags;          /* RX_F_* below */
   uint32_t reserved[3];
 } rx_options;
@@ -75,6 +76,10 @@ typedef struct {
 #define RX_F_NO_CACHE 4u     /* do not read/write the on-disk cubin cache */
 #define RX_F_NO_PREFILTER 16u /* disable the cross-regex literal prefilter: every group
                                  runs every window, gated only by Zero Block Skipping (Sec. 6) */
+#define RX_F_NO_MODEB 32u     /* never run a cluster output-gated: with the prefilter on, a
+                                 cluster runs where its first factor occurs or state flows in (ablation) */
+#define RX_F_STATS 64u        /* debug: count visited / active windows and walk-backs per rx_match and print
+                                 them to stderr (synchronises the stream; not for timing) */
 
 /* Compile n patterns (byte strings, not NUL-terminated).  On error returns
  * the status and, if err != NULL, fills it.  *out owns everything. */
@@ -97,6 +102,14 @@ uint32_t rx_kernels_per_match(const rx_program *p);
 const char *rx_program_source(const rx_program *p);
 /* Human-readable IR / per-group geometry dump (owned by p). */
 const char *rx_program_info(const rx_program *p);
+/* The prefilter's device table (host copy, owned by p; layout documented in
+ * rx_prefilter.cpp build_prefilter) and its header words hdr[12] = {smem
+ * words, log2 bits of the 4-gram Bloom filter, of the 3-gram one, of the
+ * anchor hash, offsets of the 3-gram filter, the 2-gram bitmap, the hash, the
+ * extension entries, the factor->group ranges and triples, #factors, 0}.
+ * Returns the table's size in u32 words (0: no prefilter).  For tests and
+ * analysis; matching never needs it. */
+size_t rx_prefilter_table(const rx_program *p, const uint32_t **blob, uint32_t *hdr /* [12], nullable */);
 
 typedef struct {
   uint32_t regex;

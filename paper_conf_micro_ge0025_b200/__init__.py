@@ -20,10 +20,12 @@ _lib = None
 
 RX_OK, RX_EPARSE, RX_EUNSUPPORTED, RX_ETOOBIG, RX_EJIT, RX_ECUDA, RX_EINVAL, RX_ENOMEM, RX_EOVERFLOW = range(9)
 RX_F_NO_REBALANCE, RX_F_NO_GUARDS, RX_F_NO_CACHE, RX_F_REBALANCE, RX_F_NO_PREFILTER = 1, 2, 4, 8, 16
+RX_F_NO_MODEB, RX_F_STATS = 32, 64
 
 EXPORTED = ["rx_compile", "rx_free", "rx_num_regex", "rx_num_groups", "rx_max_lookback", "rx_max_lookahead",
             "rx_boundary_bytes", "rx_program_source", "rx_program_info", "rx_match", "rx_match_chunk",
-            "rx_rematch_chunk", "rx_last_error", "rx_kernels_per_match", "rx_set_profiling", "rx_kernel_times", "rx_match_batch"]
+            "rx_rematch_chunk", "rx_last_error", "rx_kernels_per_match", "rx_set_profiling", "rx_kernel_times", "rx_match_batch",
+            "rx_prefilter_table"]
 
 
 class RxError(RuntimeError):
@@ -74,6 +76,9 @@ def load_library():
         lib.rx_program_source.restype = ctypes.c_char_p
         lib.rx_program_info.argtypes = [vp]
         lib.rx_program_info.restype = ctypes.c_char_p
+        lib.rx_prefilter_table.argtypes = [vp, ctypes.POINTER(ctypes.POINTER(ctypes.c_uint32)),
+                                           ctypes.POINTER(ctypes.c_uint32)]
+        lib.rx_prefilter_table.restype = sz
         lib.rx_match.argtypes = [vp, vp, u64, vp, ctypes.POINTER(_Output)]
         lib.rx_match.restype = ctypes.c_int
         lib.rx_match_chunk.argtypes = [vp, vp, u64, u64, u64, u64, vp, vp, ctypes.c_int, vp, ctypes.POINTER(_Output)]
@@ -173,6 +178,19 @@ class Program:
         return self._lib.rx_program_info(self._h).decode()
 
     # --- matching -----------------------------------------------------------
+    def prefilter_table(self):
+        """(blob u32 array copy, header dict) of the prefilter's device table, or None."""
+        import numpy as np
+        ptr = ctypes.POINTER(ctypes.c_uint32)()
+        hdr = (ctypes.c_uint32 * 12)()
+        n = self._lib.rx_prefilter_table(self._h, ctypes.byref(ptr), hdr)
+        if not n:
+            return None
+        blob = np.ctypeslib.as_array(ptr, shape=(n,)).copy()
+        keys = ["smem_words", "b4bits", "b3bits", "hbits", "o_b3", "o_b2", "o_ht", "o_ext", "o_fgoff", "o_fgent",
+                "nfactor"]
+        return blob, dict(zip(keys, list(hdr)[:11]))
+
     def alloc_outputs(self, length, device=None, dense=False, digests=True, match_cap=None):
         """Output buffers of rx_output.  match_cap: None = no match list;
         an int = a list of that many rx_match_t entries ({u32 regex, u32 pad,

@@ -324,7 +324,7 @@ struct RegexEmitter {
         assign(in + 2, acc, [&](int i) { return W(acc, i) + " | " + W(nw, i); });
         assign(in + 2, fr, [&](int i) { return W(nw, i); });
         os << I << "    " << fst << " = false;\n";
-        os << I << "    if (++" << it << " > RX_LOOP_CAP) { if (lane == 0) atomicOr(c.status, 1u); break; }\n";
+        os << I << "    if (++" << it << " > RX_LOOP_CAP) { if (lane == 0) atomicOr(c.o->status, 1u); break; }\n";
         os << I << "  }\n";
         assign(in + 1, nv(id), [&](int i) { return W(acc, i); });
         os << I << "}\n";
@@ -360,10 +360,15 @@ struct RegexEmitter {
       std::string R = nv(ir.outs[k]);
       std::string m;
       for (int i = 0; i < K; ++i) m += (i ? " | " : "") + ("(" + W(R, i) + " & c.cm[" + std::to_string(i) + "])");
-      os << I << "if (c.want_dense || __any_sync(RX_FULL, (" << m << ") != 0u)) {\n";
+      // walk-back runs (mode B) only compute state
+      os << I << "if (!c.walk && (c.dense || __any_sync(RX_FULL, (" << m << ") != 0u))) {\n";
       os << I << "  V<" << K << "> ov;\n";
-      for (int i = 0; i < K; ++i) os << I << "  ov.w[" << i << "] = " << W(R, i) << ";\n";
-      os << I << "  rx_emit<" << K << ">(c, " << out_member[k] << ", ov);\n";
+      os << I << "  u32 cwb = 0u;\n";
+      for (int i = 0; i < K; ++i) {
+        os << I << "  ov.w[" << i << "] = " << W(R, i) << " & c.cm[" << i << "];\n";
+        os << I << "  cwb |= (c.cm[" << i << "] != 0u ? 1u : 0u) << " << i << ";\n";
+      }
+      os << I << "  rx_emit<" << K << ">(c.o, " << out_member[k] << ", c.lane, c.word0, ov, cwb);\n";
       os << I << "}\n";
     }
   }
@@ -487,15 +492,24 @@ static void layout(const CompiledSet &cs, int &nsmax, int &nrmax) {
 // per-warp shared bytes of the literal-run scratch (frame bytes + output words)
 int lit_scratch_bytes(const CompiledSet &cs) {
   int kmax = 1;
+  bool any = false;
+  for (auto &g : cs.groups) {
+    kmax = std::max(kmax, g.K);
+    for (auto &c : g.clusters) any = any || !c.ir.lits.empty();
+  }
+  return any ? 1152 * kmax : 0;
+}
+int max_words_per_lane(const CompiledSet &cs) {
+  int kmax = 1;
   for (auto &g : cs.groups) kmax = std::max(kmax, g.K);
-  return 1152 * kmax;
+  return kmax;
 }
 
 // One relocatable compilation unit per group (NVRTC -rdc): the group's
 // traits, its program body, and the two non-inlined entry functions
 // rx_seg_<g> (pass 1 over one segment) and rx_fix_<g> (carry fix-up).
-// Compile time stays linear in the number of groups; nvJitLink links the
-// units with the kernel unit into one module.
+// Compile time stays linear in the number of groups; the CUDA driver links
+// the units with the kernel unit into one module.
 std::string emit_group_unit(CompiledSet &cs, int gi) {
   std::ostringstream os;
   os << kDevicePrelude << "\n// ===================== generated group " << gi << " =====================\n";
@@ -504,190 +518,171 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
   int G = (int)cs.groups.size();
   int sbase = 0;
   for (int h = 0; h < gi; ++h) sbase += cs.groups[h].nslots;
-  {
-    Group &g = cs.groups[gi];
-    // the group's literal runs (Op::Lit), one byte table
-    std::vector<std::vector<int>> lit_off(g.clusters.size());
-    std::string pool;
-    for (size_t ci = 0; ci < g.clusters.size(); ++ci)
-      for (auto &l : g.clusters[ci].ir.lits) {
-        lit_off[ci].push_back((int)pool.size());
-        pool += l;
+  Group &g = cs.groups[gi];
+  // the group's literal runs (Op::Lit), one byte table
+  std::vector<std::vector<int>> lit_off(g.clusters.size());
+  std::string pool;
+  for (size_t ci = 0; ci < g.clusters.size(); ++ci)
+    for (auto &l : g.clusters[ci].ir.lits) {
+      lit_off[ci].push_back((int)pool.size());
+      pool += l;
+    }
+  os << "__device__ const unsigned char rx_litb_" << gi << "[" << std::max<size_t>(pool.size(), 1) << "] = {";
+  for (size_t i = 0; i < pool.size(); ++i) os << (i ? "," : "") << (unsigned)(unsigned char)pool[i];
+  if (pool.empty()) os << "0";
+  os << "};\n";
+  os << "__device__ const int rx_rid_" << gi << "[" << g.regexes.size() << "] = {";
+  for (size_t i = 0; i < g.regexes.size(); ++i) os << (i ? "," : "") << g.regexes[i];
+  os << "};\n";
+  const int NC = (int)g.clusters.size();
+  std::vector<uint32_t> cmask(NC, 0u);
+  for (int ci = 0; ci < NC; ++ci)
+    for (int m : g.clusters[ci].members) cmask[ci] |= 1u << m;
+  // per state slot: its cluster, and its top value (the largest state it can
+  // hold: a MatchStar carry is 0/1, a forwarded advance tail a whole word)
+  // for the mode-B walk-back
+  std::vector<uint32_t> sci(std::max(g.nslots, 1), 0u), top(std::max(g.nslots, 1), 0u);
+  uint32_t calways = 0u, cbcap = 0u;
+  for (int ci = 0; ci < NC; ++ci) {
+    const Cluster &cl = g.clusters[ci];
+    if (cl.always) calways |= 1u << ci;
+    if (cl.bcap) cbcap |= 1u << ci;
+    for (auto &n : cl.ir.nodes)
+      if (n.slot >= 0) {
+        sci[cl.slot_base + n.slot] = (uint32_t)ci;
+        top[cl.slot_base + n.slot] = n.op == Op::MStar ? 1u : 0xffffffffu;
       }
-    os << "__device__ const unsigned char rx_litb_" << gi << "[" << std::max<size_t>(pool.size(), 1) << "] = {";
-    for (size_t i = 0; i < pool.size(); ++i) os << (i ? "," : "") << (unsigned)(unsigned char)pool[i];
-    if (pool.empty()) os << "0";
-    os << "};\n";
-    os << "__device__ const int rx_rid_" << gi << "[" << g.regexes.size() << "] = {";
-    for (size_t i = 0; i < g.regexes.size(); ++i) os << (i ? "," : "") << g.regexes[i];
-    os << "};\n";
-    os << "struct RxG" << gi << " {\n";
-    os << "  static constexpr int K = " << g.K << ", Lw = " << g.Lw << ", Bw = " << g.Bw << ", NS = " << g.nslots
-       << ", NR = " << g.regexes.size() << ", SBASE = " << sbase << ", NG = " << G << ", GID = " << gi
-       << ", NSMAX = " << nsmax << ";\n";
-    os << "  static DEV const int *rid() { return rx_rid_" << gi << "; }\n";
-    os << "  static constexpr unsigned ALWAYS = " << g.always << "u;\n";
-    os << "  static constexpr bool PF = " << (cs.use_pf ? "true" : "false") << ";\n";
-    os << "  static constexpr bool LIT = " << (pool.empty() ? "false" : "true") << ";\n";
-    // rmask: members whose prefilter factor occurs in the window frame
-    // (rx_prefilter); members without a factor (ALWAYS) and members carrying
-    // state into the window run regardless
-    // one out-of-line copy shared by pass 1 and both fix-up runs (code size,
-    // NVRTC time; the call costs nothing next to the body)
-    // The group's program: body() runs every factor cluster in one
-    // out-of-line function (shared by pass 1 and both fix-up runs), with
-    // the CC networks CSE'd across the clusters.  With cluster-major code
-    // generation (RX_CMAJOR_GEN=1, an experiment: DESIGN.md "Scheduling")
-    // each cluster also gets its own function cb<ci> that pass 1 runs over
-    // consecutive windows.
-    const int NC = (int)g.clusters.size();
-    const char *cmg = getenv("RX_CMAJOR_GEN");
-    const bool gen_cm = cmg && *cmg == '1';
-    std::vector<uint32_t> cmask(NC, 0u);
-    for (int ci = 0; ci < NC; ++ci)
-      for (int m : g.clusters[ci].members) cmask[ci] |= 1u << m;
-    auto emit_fn = [&](const std::string &name, int c0, int c1, bool inl = false) {
-      os << "  static __device__ " << (inl ? "__forceinline__" : "__noinline__") << " void " << name << "(Ctx<" << g.K
-         << "> &c, const u32 (&pl)[8][" << g.K
-         << "], const u32 *st, u32 *nst, const u32 rmask) {\n";
-      os << "    (void)st; (void)nst; (void)rmask;\n";
-      os << "    const u32 lane = c.lane; const int cw = (int)c.cw; (void)cw; (void)lane;\n";
-      for (int k = 0; k < 8; ++k)
-        for (int i = 0; i < g.K; ++i)
-          os << "    const u32 b" << k << "w" << i << " = pl[" << k << "][" << i << "]; (void)b" << k << "w" << i << ";\n";
-      for (int i = 0; i < g.K; ++i) os << "    const u32 vmw" << i << " = c.vm[" << i << "]; (void)vmw" << i << ";\n";
+  }
+  os << "__device__ const unsigned char rx_sci_" << gi << "[" << sci.size() << "] = {";
+  for (size_t i = 0; i < sci.size(); ++i) os << (i ? "," : "") << sci[i];
+  os << "};\n__device__ const unsigned rx_top_" << gi << "[" << top.size() << "] = {";
+  for (size_t i = 0; i < top.size(); ++i) os << (i ? "," : "") << top[i] << "u";
+  os << "};\n__device__ const unsigned rx_cm_" << gi << "[" << std::max(NC, 1) << "] = {";
+  for (int ci = 0; ci < NC; ++ci) os << (ci ? "," : "") << cmask[ci] << "u";
+  if (NC == 0) os << "0u";
+  os << "};\n";
+  os << "struct RxG" << gi << " {\n";
+  os << "  static constexpr int K = " << g.K << ", Lw = " << g.Lw << ", Bw = " << g.Bw << ", NS = " << g.nslots
+     << ", NR = " << g.regexes.size() << ", SBASE = " << sbase << ", NG = " << G << ", GID = " << gi
+     << ", NSMAX = " << nsmax << ", NC = " << NC << ";\n";
+  os << "  static DEV const int *rid() { return rx_rid_" << gi << "; }\n";
+  os << "  static constexpr unsigned ALWAYS = " << g.always << "u;    // members without a first factor\n";
+  os << "  static constexpr unsigned CALWAYS = " << calways << "u;   // clusters of them\n";
+  os << "  static constexpr unsigned CBCAP = " << cbcap << "u;     // clusters that may run output-gated\n";
+  os << "  static constexpr bool PF = " << (cs.use_pf ? "true" : "false") << ";\n";
+  os << "  static constexpr bool LIT = " << (pool.empty() ? "false" : "true") << ";\n";
+  os << "  static DEV u32 sci(int s) { return (u32)__ldg(&rx_sci_" << gi << "[s]); }\n";
+  os << "  static DEV u32 top(int s) { return __ldg(&rx_top_" << gi << "[s]); }\n";
+  os << "  static DEV u32 cmask(int ci) { return __ldg(&rx_cm_" << gi << "[ci]); }\n";
+  // The group's program: one block of code per factor cluster, entered only
+  // for the clusters in `run` (a cluster bitmask computed by the runner:
+  // prefilter hits, carried state, walk-back targets) -- the warp jumps from
+  // one active cluster to the next instead of walking past the inactive
+  // ones.  body() is the out-of-line copy shared by the walk-back and both
+  // fix-up runs; body_i is inlined into pass 1's sparse runner (the basis
+  // planes and the window context stay in registers).
+  auto emit_fn = [&](const std::string &name, bool inl) {
+    os << "  static __device__ " << (inl ? "__forceinline__" : "__noinline__") << " void " << name << "(Ctx<" << g.K
+       << "> &c, const u32 (&pl)[8][" << g.K << "], const u32 *st, u32 *nst, u32 run) {\n";
+    os << "    (void)st; (void)nst;\n";
+    os << "    const u32 lane = c.lane; const int cw = (int)c.cw; (void)cw; (void)lane;\n";
+    for (int k = 0; k < 8; ++k)
+      for (int i = 0; i < g.K; ++i)
+        os << "    const u32 b" << k << "w" << i << " = pl[" << k << "][" << i << "]; (void)b" << k << "w" << i << ";\n";
+    for (int i = 0; i < g.K; ++i) os << "    const u32 vmw" << i << " = c.vm[" << i << "]; (void)vmw" << i << ";\n";
+    os << "    while (run) {\n      const int ci = __ffs(run) - 1;\n      run &= run - 1u;\n      switch (ci) {\n";
+    for (int ci = 0; ci < NC; ++ci) {
+      const Cluster &cl = g.clusters[ci];
       std::vector<std::map<TabKey, std::string>> ccs(1);
       std::vector<std::map<std::vector<uint64_t>, std::string>> sets(1);
-      for (int ci = c0; ci < c1; ++ci) {
-        const Cluster &cl = g.clusters[ci];
-        RegexEmitter em(os, cl.ir, g.K, ci, cl.slot_base, ccs, sets);
-        em.out_member = cl.members;
-        em.lit_pool = "rx_litb_" + std::to_string(gi);
-        em.lit_off = lit_off[ci];
-        std::string run;
-        if (cl.always) {
-          run = "true";
-        } else {
-          run = "(rmask & " + std::to_string(cmask[ci]) + "u) != 0u";
-          if (cl.ir.nslots > 0) {
-            std::string pend;
-            for (int sl = 0; sl < cl.ir.nslots; ++sl) pend += (sl ? " | " : "") + em.st(sl);
-            run += " || ((" + pend + ") != 0u)";
-          }
-        }
-        // one block per factor cluster: its unguarded (shared) head and guard
-        // tests (phase 1), then its guarded bodies (phase 2) if a guard fired
-        os << "    if (" << run << ") {\n";
-        em.push();
-        std::string need = em.emit_phase1();
-        if (!need.empty()) {
-          os << "    if (" << need << ") {\n";
-          em.emit_phase2();
-          os << "    }\n";
-        }
-        em.pop();
+      RegexEmitter em(os, cl.ir, g.K, ci, cl.slot_base, ccs, sets);
+      em.out_member = cl.members;
+      em.lit_pool = "rx_litb_" + std::to_string(gi);
+      em.lit_off = lit_off[ci];
+      // its unguarded (shared) head and guard tests (phase 1), then its
+      // guarded bodies (phase 2) if a guard fired
+      os << "      case " << ci << ": {\n";
+      em.push();
+      std::string need = em.emit_phase1();
+      if (!need.empty()) {
+        os << "    if (" << need << ") {\n";
+        em.emit_phase2();
         os << "    }\n";
       }
-      os << "  }\n";
-    };
-    emit_fn("body", 0, NC);
-    // the same program inlined into pass 1's sparse runner: the basis planes
-    // and the window context stay in registers (the out-of-line call kept
-    // them in local memory, ~1.2 GB of DRAM writes per Snort-like step)
-    emit_fn("body_i", 0, NC, true);
-    if (gen_cm)
-      for (int ci = 0; ci < NC; ++ci) emit_fn("cb" + std::to_string(ci), ci, ci + 1);
-    os << "  static constexpr int NC = " << (gen_cm ? NC : 0) << ";\n";
-    os << "  static DEV u32 cmask(int ci) {\n    switch (ci) {\n";
-    for (int ci = 0; ci < NC; ++ci) os << "      case " << ci << ": return " << cmask[ci] << "u;\n";
-    os << "      default: return 0u;\n    }\n  }\n";
-    os << "  static DEV bool calways(int ci) {\n    switch (ci) {\n";
-    for (int ci = 0; ci < NC; ++ci) os << "      case " << ci << ": return " << (g.clusters[ci].always ? "true" : "false") << ";\n";
-    os << "      default: return false;\n    }\n  }\n";
-    os << "  static DEV int cslot(int ci) {  // first state slot of cluster ci (ci = NC: total)\n    switch (ci) {\n";
-    for (int ci = 0; ci < NC; ++ci) os << "      case " << ci << ": return " << g.clusters[ci].slot_base << ";\n";
-    os << "      default: return " << g.nslots << ";\n    }\n  }\n";
-    os << "  static DEV void cbody(int ci, Ctx<" << g.K << "> &c, const u32 (&pl)[8][" << g.K
-       << "], const u32 *st, u32 *nst, const u32 rmask) {\n    (void)ci; (void)c; (void)pl; (void)st; (void)nst; (void)rmask;\n";
-    if (gen_cm) {
-      os << "    switch (ci) {\n";
-      for (int ci = 0; ci < NC; ++ci) os << "      case " << ci << ": cb" << ci << "(c, pl, st, nst, rmask); break;\n";
-      os << "      default: break;\n    }\n";
+      em.pop();
+      os << "      } break;\n";
     }
-    os << "  }\n};\n";
-    const int LB = lit_scratch_bytes(cs);
-    os << "extern \"C\" __device__ __noinline__ void rx_seg_" << gi
-       << "(const RxParams &p, int seg) {\n"
-       // shared memory (rx_runtime.cpp launch() mirrors it): [wpb][3*NRMAX] u64
-       // accumulators | [wpb][4*NSMAX] u32 state | [wpb][LB] literal-run
-       // scratch | [wpb][4096] window staging (TMA) | [wpb][2] u64 mbarriers
+    os << "      default: break;\n      }\n    }\n  }\n";
+  };
+  emit_fn("body", false);
+  emit_fn("body_i", true);
+  os << "};\n";
+  // shared memory per warp (rx_runtime.cpp launch() mirrors it):
+  //   acc [3*NRMAX] u64 | RxOut | state [6*NSMAX] u32 | literal-run scratch [LB]
+  //   | window staging [TB] (TMA) | mbarrier u64
+  const int LB = lit_scratch_bytes(cs), TB = 1024 * max_words_per_lane(cs);
+  const int ACC = (24 * nrmax + 15) & ~15, OUTB = 96, STB = ((24 * nsmax) + 15) & ~15;
+  const int PER = ACC + OUTB + STB + LB + TB + 16;
+  os << "static_assert(sizeof(RxOut) <= " << OUTB << ", \"RxOut layout\");\n";
+  os << "#define RX_WARP_SMEM_" << gi << " " << PER << "\n";
+  os << "extern \"C\" __device__ __noinline__ void rx_seg_" << gi << "(const RxParams &p, int seg) {\n"
+     << "  extern __shared__ __align__(16) u64 rx_smem[];\n"
+     << "  const int warp = threadIdx.x >> 5;\n"
+     << "  unsigned char *base = reinterpret_cast<unsigned char *>(rx_smem) + (size_t)warp * " << PER << ";\n"
+     << "  u64 *acc = reinterpret_cast<u64 *>(base);\n"
+     << "  RxOut *o = reinterpret_cast<RxOut *>(base + " << ACC << ");\n"
+     << "  u32 *st = reinterpret_cast<u32 *>(base + " << ACC + OUTB << ");\n"
+     << "  unsigned char *lb = base + " << ACC + OUTB + STB << ";\n"
+     << "  unsigned char *tb = base + " << ACC + OUTB + STB + LB << ";\n"
+     << "  u64 *bar = reinterpret_cast<u64 *>(base + " << ACC + OUTB + STB + LB + TB << ");\n"
+     << "  (void)tb; (void)bar;\n";
+  if (cs.use_pf)
+    os << "  if (p.pf_on) { rx_run_segment_pf<RxG" << gi << ">(p, seg, o, acc, st, tb, bar, lb); return; }\n";
+  os << "  rx_run_segment_dense<RxG" << gi << ">(p, seg, o, acc, st, lb);\n}\n";
+  if (g.nslots > 0)
+    os << "extern \"C\" __device__ __noinline__ void rx_fix_" << gi << "(const RxParams &p, int seg) {\n"
        << "  extern __shared__ __align__(16) u64 rx_smem[];\n"
-       << "  const int warp = threadIdx.x >> 5, wpb = blockDim.x >> 5;\n"
-       << "  u64 *acc = rx_smem + warp * (3 * " << nrmax << ");\n"
-       << "  u32 *st0 = reinterpret_cast<u32 *>(rx_smem + wpb * (3 * " << nrmax << "));\n"
-       << "  unsigned char *lb0 = reinterpret_cast<unsigned char *>(st0 + ((wpb * (4 * " << nsmax
-       << ") + 3) & ~3));\n"
-       << "  unsigned char *tb0 = lb0 + wpb * " << LB << ";\n"
-       << "  u64 *bars = reinterpret_cast<u64 *>(tb0 + wpb * 4096) + 2 * warp;\n"
-       << "  rx_run_segment<RxG" << gi << ">(p, seg, acc, st0 + warp * (4 * " << nsmax
-       << "), tb0 + warp * 4096, bars, lb0 + warp * " << LB << ");\n}\n";
-    if (g.nslots > 0)
-      os << "extern \"C\" __device__ __noinline__ void rx_fix_" << gi << "(const RxParams &p, int seg) {\n"
-         << "  extern __shared__ __align__(16) u64 rx_smem[];\n"
-         << "  const int warp = threadIdx.x >> 5, wpb = blockDim.x >> 5;\n"
-         << "  u32 *st0 = reinterpret_cast<u32 *>(rx_smem + wpb * (3 * " << nrmax << "));\n"
-         << "  unsigned char *lb0 = reinterpret_cast<unsigned char *>(st0 + ((wpb * (4 * " << nsmax
-         << ") + 3) & ~3));\n"
-         << "  rx_fixup_group<RxG" << gi << ">(p, rx_smem + warp * (3 * " << nrmax << "), st0 + warp * (4 * " << nsmax
-         << "), lb0 + warp * " << LB << ", seg);\n}\n";
-  }
+       << "  const int warp = threadIdx.x >> 5;\n"
+       << "  unsigned char *base = reinterpret_cast<unsigned char *>(rx_smem) + (size_t)warp * " << PER << ";\n"
+       << "  rx_fixup_group<RxG" << gi << ">(p, reinterpret_cast<RxOut *>(base + " << ACC
+       << "), reinterpret_cast<u64 *>(base), reinterpret_cast<u32 *>(base + " << ACC + OUTB << "), base + "
+       << ACC + OUTB + STB << ", seg);\n}\n";
   return os.str();
 }
 
-// The kernel unit: rx_pass1 (warp -> (segment, group), groups of one
-// segment interleaved so that they read the same input region together)
-// and rx_fixup (one warp per stateful group).
+// per-warp shared bytes of pass 1 / fix-up (must match emit_group_unit)
+size_t warp_smem_bytes(const CompiledSet &cs) {
+  int nsmax, nrmax;
+  layout(cs, nsmax, nrmax);
+  const int LB = lit_scratch_bytes(cs), TB = 1024 * max_words_per_lane(cs);
+  return (size_t)(((24 * nrmax + 15) & ~15) + 96 + (((24 * nsmax) + 15) & ~15) + LB + TB + 16);
+}
+
+// The kernel unit: rx_pass1 (a CTA of 16 warps runs one group over 16
+// consecutive segments), rx_prefilter, rx_fixup (phase 1: one warp per
+// (group, segment); phase 2 and rematch: one warp per group).
 std::string emit_kernel_unit(CompiledSet &cs) {
   std::ostringstream os;
   os << kDevicePrelude << "\n// ===================== kernels =====================\n";
-  int nsmax, nrmax;
-  layout(cs, nsmax, nrmax);
   int G = (int)cs.groups.size();
-  os << "#define RX_NG " << G << "\n#define RX_NSMAX " << nsmax << "\n#define RX_NRMAX " << nrmax << "\n";
+  os << "#define RX_NG " << G << "\n";
   for (int gi = 0; gi < G; ++gi) {
     os << "extern \"C\" __device__ void rx_seg_" << gi << "(const RxParams &p, int seg);\n";
     if (cs.groups[gi].nslots > 0) os << "extern \"C\" __device__ void rx_fix_" << gi << "(const RxParams &p, int seg);\n";
   }
-  int g_begin = 0;
-  // pass 1: one CTA of 16 warps (the whole SM's register file) runs one
-  // group over 16 consecutive segments in lockstep, so the SM's instruction
-  // caches hold one program at a time
   os << "\nextern \"C\" __global__ void __launch_bounds__(512, 1) rx_pass1(const RxParams p) {\n"
         "  const int warp = threadIdx.x >> 5;\n"
         "  const int wpb = blockDim.x >> 5;\n"
         "  const int cpg = (p.nseg_max + wpb - 1) / wpb;  // CTAs per group\n"
         "  const int g = (int)(blockIdx.x / cpg);\n"
         "  const long long seg = (long long)(blockIdx.x % cpg) * wpb + warp;\n"
-        "  if (p.task_ctr) {\n"
-        "    // dynamic: every warp pulls (group, segment) tasks, group-major, from\n"
-        "    // one counter until they run out (load balance under zero skipping)\n"
-        "    const long long ntask = (long long)RX_NG * p.nseg_max;\n"
-        "    for (;;) {\n"
-        "      unsigned long long t = 0;\n"
-        "      if ((threadIdx.x & 31) == 0) t = atomicAdd(p.task_ctr, 1ull);\n"
-        "      t = __shfl_sync(RX_FULL, t, 0);\n"
-        "      if ((long long)t >= ntask) return;\n"
-        "      const int tg = (int)(t / p.nseg_max), ts = (int)(t % p.nseg_max);\n"
-        "      switch (tg) {\n";
-  for (int gi = 0; gi < G; ++gi) os << "        case " << gi << ": rx_seg_" << gi << "(p, ts); break;\n";
-  os << "        default: break;\n      }\n      __syncwarp();\n    }\n  }\n";
-  os << "  if (g >= RX_NG) return;\n"
+        "  if (g >= RX_NG) return;\n"
         "  switch (g) {\n";
   for (int gi = 0; gi < G; ++gi) os << "    case " << gi << ": rx_seg_" << gi << "(p, (int)seg); break;\n";
   os << "    default: break;\n  }\n}\n";
   if (cs.use_pf)
-    os << "\nextern \"C\" __global__ void __launch_bounds__(512, 1) rx_prefilter(const RxParams p) {\n"
-          "  rx_prefilter_run(p, RX_NG, p.pf_tab_smem != 0);\n}\n";
+    os << "\nextern \"C\" __global__ void __launch_bounds__(256, 3) rx_prefilter(const RxParams p) {\n"
+          "  rx_prefilter_run(p, RX_NG);\n}\n";
   os << "\nextern \"C\" __global__ void __launch_bounds__(128) rx_fixup(const RxParams p) {\n"
         "  const int warp = threadIdx.x >> 5;\n"
         "  const int wpb = blockDim.x >> 5;\n"
@@ -698,7 +693,7 @@ std::string emit_kernel_unit(CompiledSet &cs) {
         "  if (g >= RX_NG) return;\n"
         "  switch ((int)g) {\n";
   for (int gi = 0; gi < G; ++gi)
-    if (cs.groups[g_begin + gi].nslots > 0) os << "    case " << gi << ": rx_fix_" << gi << "(p, seg); break;\n";
+    if (cs.groups[gi].nslots > 0) os << "    case " << gi << ": rx_fix_" << gi << "(p, seg); break;\n";
   os << "    default: break;\n  }\n}\n";
   return os.str();
 }

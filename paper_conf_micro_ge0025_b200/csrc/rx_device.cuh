@@ -21,6 +21,11 @@
 //    bit transpose per 32 bytes;
 //  * zero-block skipping uses __any_sync votes (warp-uniform branches, the
 //    paper's block-wide atomicOr of P:L372 at warp scope);
+//  * a cross-regex prefilter (rx_prefilter_run) decides which clusters of a
+//    group run in which windows: mode A -- where a first factor occurs or
+//    state flows in; mode B -- only where an output factor occurs, with the
+//    state the window needs reconstructed by a convergence walk-back
+//    (rx_walk_back);
 //  * the epilogue popcounts committed words (REDUX), folds positions into
 //    additive digests and optionally stores the dense match bitstreams.
 typedef unsigned int u32;
@@ -42,36 +47,44 @@ DEV u32 rx_lane() {
 }
 
 // ---------------------------------------------------------------------------
+// emission context: per-warp, in shared memory (the out-of-line epilogue
+// reads it there instead of taking a large struct by value)
+// ---------------------------------------------------------------------------
+struct RxOut {
+  u64 *acc;         // per-warp shared accumulators [NR][3] (count, d1, d2)
+  u32 *dense;       // nullable
+  u64 pitch;
+  i64 gofs;         // global position of chunk position 0
+  u64 sign;         // 1 (add) or 2^64-1 (subtract; fix-up pass)
+  const int *rid;   // group member -> global regex id
+  u32 *status;
+  u64 *mlist;       // nullable: compacted match list, {regex, pos} pairs (rx_match_t)
+  u64 mcap;
+  u64 *mtotal;
+  u32 *fold;        // fix-up only: [NR][K] output words of the "old" run (match-list delta)
+  int want_digest, want_dense;
+};
+
 // window context (scalars only: the 8 basis streams live in a register array
 // of the segment loop and are passed to the body separately)
-// ---------------------------------------------------------------------------
 template <int K>
 struct Ctx {
   u32 vm[K];    // positions holding real stream bytes
   u32 cm[K];    // committed positions of this window inside [0, len)
   u32 lane;
   u32 cw;       // committed words of this window
-  u64 *acc;     // per-warp shared accumulators [NR][3] (count, d1, d2)
-  u32 *dense;   // nullable
-  u64 pitch;
   i64 word0;    // chunk word index of local word 0
-  i64 gofs;     // global position of chunk position 0
-  u64 sign;     // 1 (add) or 2^64-1 (subtract; fix-up pass)
-  bool want_digest, want_dense;
-  const int *rid;  // group member -> global regex id
-  u32 *status;
-  u64 *mlist;      // nullable: compacted match list, {regex, pos} pairs (rx_match_t)
-  u64 mcap;
-  u64 *mtotal;
-  u32 *fold;       // fix-up only: [NR][K] output words of the "old" run (match-list delta)
+  RxOut *o;     // shared memory
   unsigned char *wb;  // nullable (groups without literal runs): the frame's bytes, frame position f at wb[f]
   u32 *ob;            // literal-run output scratch, 32*K words (per warp)
+  bool walk;          // state-only run (mode-B walk-back): no output
+  bool dense;         // dense output requested (mirrors o->want_dense)
 };
 
 // ---------------------------------------------------------------------------
 // epilogue (called only when the output has a set bit in the committed
 // range, or when dense output is requested): popcount -> REDUX, digests,
-// dense store
+// dense store, match list
 // ---------------------------------------------------------------------------
 DEV u64 rx_splitmix64(u64 x) {
   u64 z = x + 0x9E3779B97F4A7C15ull;
@@ -89,84 +102,82 @@ DEV u64 rx_warp_sum64(u64 v) {
 // Compacted match list (rx_output.d_matches): every set bit of the committed
 // words becomes one {regex, global position} entry; a warp reserves its slots
 // with one atomicAdd and each lane writes its own bits after an exclusive
-// prefix sum.  The fix-up's "old" run (sign = -1) records its words in c.fold
+// prefix sum.  The fix-up's "old" run (sign = -1) records its words in o->fold
 // and the "new" run lists only the bits the old one lacked: match sets are
 // monotone in the incoming state (every operation on state streams is AND /
 // OR / Advance / add-with-carry of a marker into a class), so new covers old;
 // a violation is flagged in status bit 2 instead of being silently dropped.
 template <int K>
-DEV void rx_emit_list(const Ctx<K> &c, int r, const u32 (&m)[K]) {
+DEV void rx_emit_list(const RxOut *o, int r, u32 lane, i64 word0, const u32 (&m)[K]) {
   u32 mm[K];
   u32 cnt = 0;
   bool lost = false;
 #pragma unroll
   for (int i = 0; i < K; ++i) {
-    if (c.fold && c.sign == ~0ull) {
-      c.fold[r * K + i] = m[i];
+    if (o->fold && o->sign == ~0ull) {
+      o->fold[r * K + i] = m[i];
       mm[i] = 0u;
-    } else if (c.fold) {
-      lost = lost || (c.fold[r * K + i] & ~m[i]) != 0u;
-      mm[i] = m[i] & ~c.fold[r * K + i];
+    } else if (o->fold) {
+      lost = lost || (o->fold[r * K + i] & ~m[i]) != 0u;
+      mm[i] = m[i] & ~o->fold[r * K + i];
     } else {
       mm[i] = m[i];
     }
     cnt += __popc(mm[i]);
   }
-  if (lost) atomicOr(c.status, 4u);
+  if (lost) atomicOr(o->status, 4u);
   u32 incl = cnt;
 #pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    const u32 t = __shfl_up_sync(RX_FULL, incl, o);
-    if (c.lane >= (u32)o) incl += t;
+  for (int s = 1; s < 32; s <<= 1) {
+    const u32 t = __shfl_up_sync(RX_FULL, incl, s);
+    if (lane >= (u32)s) incl += t;
   }
   const u32 tot = __shfl_sync(RX_FULL, incl, 31);
   if (tot == 0u) return;
   u64 base = 0;
-  if (c.lane == 0) base = atomicAdd(c.mtotal, (u64)tot);
+  if (lane == 0) base = atomicAdd(o->mtotal, (u64)tot);
   base = __shfl_sync(RX_FULL, base, 0) + (incl - cnt);
-  const u64 reg = (u64)(u32)c.rid[r];
+  const u64 reg = (u64)(u32)o->rid[r];
 #pragma unroll
   for (int i = 0; i < K; ++i) {
     u32 b = mm[i];
-    const i64 wpos = c.gofs + (c.word0 + (i64)(c.lane * K + i)) * 32;
+    const i64 wpos = o->gofs + (word0 + (i64)(lane * K + i)) * 32;
     while (b) {
       const int t = __ffs(b) - 1;
       b &= b - 1u;
-      if (base < c.mcap) {
-        c.mlist[2 * base] = reg;
-        c.mlist[2 * base + 1] = (u64)(wpos + t);
+      if (base < o->mcap) {
+        o->mlist[2 * base] = reg;
+        o->mlist[2 * base + 1] = (u64)(wpos + t);
       }
       ++base;
     }
   }
 }
 
+// m: the output words already masked to the committed positions; cwb: bit i
+// set if word i of this lane is committed (dense stores)
 template <int K>
-__device__ __noinline__ void rx_emit(const Ctx<K> c, int r, const V<K> v) {
-  u32 m[K];
+__device__ __noinline__ void rx_emit(const RxOut *o, int r, u32 lane, i64 word0, const V<K> m, u32 cwb) {
   u32 any = 0u;
 #pragma unroll
-  for (int i = 0; i < K; ++i) {
-    m[i] = v.w[i] & c.cm[i];
-    any |= m[i];
-  }
-  if (c.want_dense) {
-    u32 *row = c.dense + (u64)c.rid[r] * c.pitch;
+  for (int i = 0; i < K; ++i) any |= m.w[i];
+  if (o->want_dense) {
+    u32 *row = o->dense + (u64)o->rid[r] * o->pitch;
 #pragma unroll
     for (int i = 0; i < K; ++i)
-      if (c.cm[i] != 0u) row[c.word0 + (i64)(c.lane * K + i)] = m[i];
+      if ((cwb >> i) & 1u) row[word0 + (i64)(lane * K + i)] = m.w[i];
   }
   if (!__any_sync(RX_FULL, any != 0u)) return;
   u32 cnt = 0;
 #pragma unroll
-  for (int i = 0; i < K; ++i) cnt += __popc(m[i]);
+  for (int i = 0; i < K; ++i) cnt += __popc(m.w[i]);
   const u32 tot = __reduce_add_sync(RX_FULL, cnt);
   u64 d1 = 0, d2 = 0;
-  if (c.want_digest) {
+  if (o->want_digest) {
 #pragma unroll
     for (int i = 0; i < K; ++i) {
-      u32 b = m[i];
-      const i64 base = c.gofs + (c.word0 + (i64)(c.lane * K + i)) * 32;
+      u32 b = m.w[i];
+      const i64 base = o->gofs + (word0 + (i64)(lane * K + i)) * 32;
       while (b) {
         const int t = __ffs(b) - 1;
         b &= b - 1u;
@@ -178,12 +189,17 @@ __device__ __noinline__ void rx_emit(const Ctx<K> c, int r, const V<K> v) {
     d1 = rx_warp_sum64(d1);
     d2 = rx_warp_sum64(d2);
   }
-  if (c.lane == 0) {
-    c.acc[3 * r + 0] += c.sign * (u64)tot;
-    c.acc[3 * r + 1] += c.sign * d1;
-    c.acc[3 * r + 2] += c.sign * d2;
+  if (lane == 0) {
+    o->acc[3 * r + 0] += o->sign * (u64)tot;
+    o->acc[3 * r + 1] += o->sign * d1;
+    o->acc[3 * r + 2] += o->sign * d2;
   }
-  if (c.mtotal) rx_emit_list<K>(c, r, m);
+  if (o->mtotal) {
+    u32 mm[K];
+#pragma unroll
+    for (int i = 0; i < K; ++i) mm[i] = m.w[i];
+    rx_emit_list<K>(o, r, lane, word0, mm);
+  }
 }
 
 // ---------------------------------------------------------------------------
@@ -287,78 +303,33 @@ struct RxParams {
   int aligned;              // in is 16-byte aligned
   int mode;                 // 0 = pass 1, 1 = fix-up with stored segment states, 2 = rematch
   int accumulate;           // counts/digests are added to (else the host zeroed them)
-  int lockstep;             // pass 1: one CTA barrier per window (warps of a group stay in step)
-  // cross-regex prefilter (rx_prefilter below)
-  // one table blob (rx_prefilter.cpp build_prefilter), u32 words:
-  //   [0,2048) l1 bigram bitmap | [2048,4096) rank: set bits before word i |
-  //   bsid[nb]: shapes indexed by each set bigram (shape = 3*(k-2) + d) |
-  //   htab[2 << hbits]: {gram, fid << 8 | shape << 1 | 1} | fgoff[nf+1] |
-  //   fgent[2*nfe]: {group, member mask}
+  int modeb;                // mode B allowed (plain rx_match: no chunk state in/out)
+  // cross-regex prefilter (rx_prefilter_run below; rx_prefilter.cpp
+  // build_prefilter documents the table blob)
   const u32 *pf_tab;
-  u32 pf_words;             // blob size
-  u32 pf_o_ent, pf_o_fgoff, pf_o_fgent;  // word offsets: hash table, factor -> group ranges, pairs
-  u32 pf_hbits;             // log2 hash slots
-  int pf_tab_smem;          // the whole blob is staged in shared memory
-  u32 *pf_gbits;            // [NG][ntiles]: bit b of word t = factor of the group in block 32t+b
-  u32 *pf_mmask;            // [NG][32*ntiles]: members of the group whose factor occurs in the block
-                            // (written only where non-zero: read only where the pf_gbits bit is set)
+  u32 pf_words, pf_smem_words;
+  u32 pf_b4bits, pf_b3bits, pf_hbits;
+  u32 pf_o_b3, pf_o_b2, pf_o_ht, pf_o_ext, pf_o_fgoff, pf_o_fgent;
+  u32 *pf_gbits;            // [NG][ntiles]: bit b of word t = a factor of the group occurs in block 32t+b
+  u32 *pf_mmask;            // [NG][32*ntiles]: members whose FIRST factor occurs in the block
+  u32 *pf_omask;            // [NG][32*ntiles]: members whose OUTPUT factor occurs in the block
+                            // (both written wherever a pf_gbits bit is set)
+  u32 *pf_cnt;              // [NG][32][2]: blocks with a first / output factor hit per member (mode choice)
   i64 pf_ntiles;
   int pf_on;
-  int pf_aligned;           // in + avail_lo is 16-byte aligned
-  u64 *stats;               // nullable: debug counters (RX_STATS=1), see rx_run_segment_pf
-  int dbg;                  // timing experiments only (RX_DBG): 1 = skip every window, 2 = no body
+  u64 *stats;               // nullable: counters (RX_F_STATS), see rx_run_segment_pf
   u64 *matches;             // nullable: rx_match_t[match_cap] as u64 pairs {regex, pos}
   u64 match_cap;
   u64 *match_total;         // u64: matches found (may exceed match_cap)
-  int fix_phase;            // mode 1: 0 = serial fix-up, 1 = parallel per segment, 2 = serial remainder
+  int fix_phase;            // mode 1: 1 = parallel per segment, 2 = serial remainder
   u32 *seg_fix;             // [nseg_max][G][NSMAX]: phase-1 end state of a segment that did not converge
   u32 *seg_nc;              // [nseg_max][G]: that segment did not converge in phase 1
-  u64 *task_ctr;            // pass 1: non-null = persistent warps pull (group, segment) tasks from it
-  int cmajor;               // sparse pass 1 runs cluster by cluster (rx_run_segment_cm)
-  int cm_sync;              // ... with one CTA barrier per cluster (static task map only)
 };
 
-template <int K> DEV void rx_load_window(const RxParams &p, Ctx<K> &c, u32 (&pl)[8][K], i64 fword) {
-#pragma unroll
-  for (int i = 0; i < K; ++i) {
-    const i64 wi = fword + (i64)(c.lane * K + i);
-    const i64 pos = wi * 32;
-    u32 x[8];
-    if (p.aligned && pos >= p.avail_lo && pos + 32 <= p.avail_hi) {
-      const uint4 *q = reinterpret_cast<const uint4 *>(p.in + pos);
-      const uint4 a = __ldg(q), b = __ldg(q + 1);
-      x[0] = a.x; x[1] = a.y; x[2] = a.z; x[3] = a.w;
-      x[4] = b.x; x[5] = b.y; x[6] = b.z; x[7] = b.w;
-    } else {
-#pragma unroll
-      for (int j = 0; j < 8; ++j) x[j] = 0u;
-      for (int j = 0; j < 32; ++j) {
-        const i64 ps = pos + j;
-        if (ps >= p.avail_lo && ps < p.avail_hi) x[j >> 2] |= (u32)p.in[ps] << (8 * (j & 3));
-      }
-    }
-    u32 t[8];
-    rx_transpose32(x, t);
-#pragma unroll
-    for (int k = 0; k < 8; ++k) pl[k][i] = t[k];
-    // valid-data mask
-    const i64 lo = p.valid_lo - pos, hi = p.valid_hi - pos;  // valid bits [lo, hi) of this word
-    u32 m;
-    if (lo <= 0 && hi >= 32) m = RX_FULL;
-    else if (hi <= 0 || lo >= 32) m = 0u;
-    else {
-      const u32 a = lo <= 0 ? RX_FULL : (RX_FULL << (u32)lo);
-      const u32 b = hi >= 32 ? RX_FULL : (RX_FULL >> (u32)(32 - hi));
-      m = a & b;
-    }
-    c.vm[i] = m;
-  }
-}
-
 // split prologue (software pipelining): rx_fetch issues the 128-bit loads of
-// a window into registers, rx_unpack transposes them one window later.
-// Interior windows (all bytes readable and valid, 16-byte aligned) take the
-// straight path; edge windows go through an out-of-line byte loader.
+// a window into registers, rx_unpack transposes them.  Interior windows (all
+// bytes readable and valid, 16-byte aligned) take the straight path; edge
+// windows go through an out-of-line byte loader.
 struct RxW8 {
   u32 v[8];
 };
@@ -453,33 +424,39 @@ DEV i64 rx_div_up(i64 a, i64 b) { return (a + b - 1) / b; }
 
 template <class G> DEV void rx_flush(const RxParams &p, const Ctx<G::K> &c) {
   __syncwarp();
+  const u64 *acc = c.o->acc;
   for (int r = (int)c.lane; r < G::NR; r += 32) {
     const int gr = G::rid()[r];
-    if (c.acc[3 * r]) atomicAdd(&p.counts[gr], c.acc[3 * r]);
+    if (acc[3 * r]) atomicAdd(&p.counts[gr], acc[3 * r]);
     if (p.digests) {
-      if (c.acc[3 * r + 1]) atomicAdd(&p.digests[2 * gr], c.acc[3 * r + 1]);
-      if (c.acc[3 * r + 2]) atomicAdd(&p.digests[2 * gr + 1], c.acc[3 * r + 2]);
+      if (acc[3 * r + 1]) atomicAdd(&p.digests[2 * gr], acc[3 * r + 1]);
+      if (acc[3 * r + 2]) atomicAdd(&p.digests[2 * gr + 1], acc[3 * r + 2]);
     }
   }
 }
 
-template <class G> DEV void rx_ctx_init(const RxParams &p, Ctx<G::K> &c, u64 *acc, unsigned char *lb) {
+template <class G> DEV void rx_ctx_init(const RxParams &p, Ctx<G::K> &c, RxOut *o, u64 *acc, unsigned char *lb) {
   c.lane = rx_lane();
-  c.acc = acc;
-  c.dense = p.dense;
-  c.pitch = p.pitch;
-  c.gofs = p.gofs;
-  c.sign = 1ull;
-  c.want_digest = p.digests != nullptr;
-  c.want_dense = p.dense != nullptr;
-  c.rid = G::rid();
-  c.status = p.status;
-  c.mlist = p.matches;
-  c.mcap = p.match_cap;
-  c.mtotal = p.match_total;
-  c.fold = nullptr;
+  c.o = o;
+  c.walk = false;
+  c.dense = p.dense != nullptr;
   c.wb = G::LIT ? lb : nullptr;
   c.ob = G::LIT ? reinterpret_cast<u32 *>(lb + 1024 * G::K) : nullptr;
+  if (c.lane == 0) {
+    o->acc = acc;
+    o->dense = p.dense;
+    o->pitch = p.pitch;
+    o->gofs = p.gofs;
+    o->sign = 1ull;
+    o->want_digest = p.digests != nullptr;
+    o->want_dense = p.dense != nullptr;
+    o->rid = G::rid();
+    o->status = p.status;
+    o->mlist = p.matches;
+    o->mcap = p.match_cap;
+    o->mtotal = p.match_total;
+    o->fold = nullptr;
+  }
   for (int r = (int)c.lane; r < 3 * G::NR; r += 32) acc[r] = 0ull;
   __syncwarp();
 }
@@ -504,7 +481,7 @@ DEV bool rx_state_eq(const u32 *a, const u32 *b, int n, u32 lane) {
 // ---------------------------------------------------------------------------
 // TMA (bulk async copy) staging of window bytes: one elected lane copies the
 // next window's 1024*K contiguous bytes global -> shared memory, completion
-// tracked by an mbarrier (transaction bytes); double-buffered per warp.
+// tracked by an mbarrier (transaction bytes).
 // ---------------------------------------------------------------------------
 DEV u32 rx_smem_addr(const void *p) { return (u32)__cvta_generic_to_shared(p); }
 DEV void rx_mbar_init(u64 *bar, u32 count) {
@@ -533,120 +510,52 @@ DEV void rx_mbar_wait(u64 *bar, u32 phase) {
   }
 }
 
-// Runs one group (traits G) over one segment (pass 1).  Windows of groups
-// with K <= 2 are staged through shared memory by TMA bulk copies issued
-// one window ahead; wider groups prefetch into registers.
-template <class G> DEV void rx_run_segment_pf(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *lb);
-template <class G>
-DEV void rx_run_segment_pf_staged(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *tbuf, u64 *bar,
-                                  unsigned char *lb);
-template <class G>
-DEV void rx_run_segment_cm(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *tbuf, u64 *bar,
-                           unsigned char *lb);
+// ---------------------------------------------------------------------------
+// cluster masks (bit ci = the group's factor cluster ci; G::cmask(ci) = its
+// members).  The body runs exactly the clusters of its `run` mask.
+// ---------------------------------------------------------------------------
+template <class G> DEV u32 rx_all_clusters() { return G::NC >= 32 ? RX_FULL : ((1u << G::NC) - 1u); }
+// clusters with a member in `members` (lane ci looks at cluster ci)
+template <class G> DEV u32 rx_clusters_of(u32 members, u32 lane) {
+  const bool hit = (int)lane < G::NC && (G::cmask((int)lane) & members) != 0u;
+  return __ballot_sync(RX_FULL, hit);
+}
+// clusters holding a non-zero state word
+template <class G> DEV u32 rx_pend_clusters(const u32 *st, u32 lane) {
+  u32 pc = 0u;
+  for (int s = (int)lane; s < G::NS; s += 32)
+    if (st[s] != 0u) pc |= 1u << G::sci(s);
+  return __reduce_or_sync(RX_FULL, pc);
+}
+// clusters to run in a window: a prefilter hit of a member (rmask), or --
+// mode A only (not in bmc) -- carried state or no factor at all
+template <class G> DEV u32 rx_run_clusters(u32 rmask, u32 bmc, u32 pendc, u32 lane) {
+  const int ci = (int)lane;
+  bool r = false;
+  if (ci < G::NC) {
+    const u32 bit = 1u << ci;
+    r = (G::cmask(ci) & rmask) != 0u || (!(bmc & bit) && (((G::CALWAYS | pendc) & bit) != 0u));
+  }
+  return __ballot_sync(RX_FULL, r);
+}
 
+// ---------------------------------------------------------------------------
+// Dense pass 1 (no prefilter: RX_F_NO_PREFILTER or no factor at all): every
+// window of the segment runs the group's whole program, gated only by the
+// zero-block guards inside it (Sec. 6).  All warps of the CTA run this group
+// in lockstep (one barrier per window) so that the SM fetches each line of
+// the group's straight-line program once for all of them.
+// ---------------------------------------------------------------------------
 template <class G>
-DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *tbuf, u64 *bars,
-                        unsigned char *lb) {
+DEV void rx_run_segment_dense(const RxParams &p, int seg, RxOut *o, u64 *acc, u32 *sst, unsigned char *lb) {
   constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS;
-  constexpr u32 WB = 1024u * K;  // window bytes
-  if constexpr (G::PF) {
-    (void)WB;
-    if (K <= 4 && !p.lockstep && !p.dbg && p.cmajor && G::NC > 0)
-      rx_run_segment_cm<G>(p, seg, acc, sst, tbuf, bars, lb);
-    else if (K <= 4 && !p.lockstep && !p.dbg) rx_run_segment_pf_staged<G>(p, seg, acc, sst, tbuf, bars, lb);
-    else rx_run_segment_pf<G>(p, seg, acc, sst, lb);
-    return;
-  }
-  if constexpr (K <= 2) {
-    const i64 len_words = rx_div_up(p.len, 32);
-    const i64 nwin = rx_div_up(len_words, Bw);
-    const i64 w_begin = (i64)seg * p.sw;
-    const bool live = w_begin < nwin || seg == 0;
-    const i64 w_end = !live ? w_begin : (w_begin + p.sw < nwin ? w_begin + p.sw : nwin);
-    Ctx<K> c;
-    rx_ctx_init<G>(p, c, acc, lb);
-    u32 pl[8][K];
-    u32 xr[K][8];
-    u32 *st = sst, *nst = sst + G::NSMAX;
-    for (int s = (int)c.lane; s < NS; s += 32) st[s] = (seg == 0 && p.st_in) ? p.st_in[G::SBASE + s] : 0u;
-    if (c.lane == 0) {
-      rx_mbar_init(&bars[0], 1);
-      rx_mbar_init(&bars[1], 1);
-    }
-    __syncwarp();
-    const RxRange ir = rx_interior(p);
-    const bool lockstep = p.lockstep != 0;
-    bool issued0 = false, issued1 = false;
-    u32 ph0 = 0, ph1 = 0;
-    if (w_begin < w_end) {
-      const i64 f0 = w_begin * Bw - Lw;
-      if (f0 >= ir.lo && f0 + 32 * K <= ir.hi) {
-        if (c.lane == 0) rx_bulk_load(tbuf, p.in + f0 * 32, WB, &bars[0]);
-        issued0 = true;
-      }
-    }
-    for (int i = 0; i < p.sw; ++i) {
-      const i64 w = w_begin + i;
-      const int b = i & 1;
-      if (w < w_end) {
-        const i64 cstart = w * Bw;
-        const i64 fword = cstart - Lw;
-        c.cw = (u32)((len_words - cstart) < Bw ? (len_words - cstart) : Bw);
-        c.word0 = fword;
-        const bool staged = b ? issued1 : issued0;
-        if (staged) {
-          rx_mbar_wait(&bars[b], b ? ph1 : ph0);
-          if (b) { ph1 ^= 1u; issued1 = false; } else { ph0 ^= 1u; issued0 = false; }
-          const uint4 *q = reinterpret_cast<const uint4 *>(tbuf + b * WB + c.lane * (32u * K));
-#pragma unroll
-          for (int k = 0; k < K; ++k) {
-            const uint4 a0 = q[2 * k], a1 = q[2 * k + 1];
-            xr[k][0] = a0.x; xr[k][1] = a0.y; xr[k][2] = a0.z; xr[k][3] = a0.w;
-            xr[k][4] = a1.x; xr[k][5] = a1.y; xr[k][6] = a1.z; xr[k][7] = a1.w;
-          }
-        } else {
-          rx_fetch<K>(p, ir, c.lane, xr, fword);
-        }
-        // stage the next window into the other buffer (read by every lane
-        // one window ago, released by the barrier that ended it)
-        if (w + 1 < w_end) {
-          const i64 nf = fword + Bw;
-          if (nf >= ir.lo && nf + 32 * K <= ir.hi) {
-            __syncwarp();
-            if (c.lane == 0) rx_bulk_load(tbuf + (b ^ 1) * WB, p.in + nf * 32, WB, &bars[b ^ 1]);
-            if (b) issued0 = true; else issued1 = true;
-          }
-        }
-        rx_unpack<K>(p, ir, c, xr, pl, fword);
-        rx_commit_mask(p, ir, c, Lw, fword);
-        if (NS > 0) rx_state_zero(nst, NS, c.lane);
-        G::body(c, pl, st, nst, ~0u);
-        u32 *t = st;
-        st = nst;
-        nst = t;
-        __syncwarp();
-      }
-      if (lockstep) __syncthreads();
-    }
-    if (!live) return;
-    if (NS > 0) {
-      u32 *dst = p.seg_state + ((i64)seg * G::NG + G::GID) * G::NSMAX;
-      for (int s = (int)c.lane; s < NS; s += 32) dst[s] = st[s];
-      if (p.st_out && w_end == nwin)
-        for (int s = (int)c.lane; s < NS; s += 32) p.st_out[G::SBASE + s] = st[s];
-    }
-    rx_flush<G>(p, c);
-    return;
-  }
-  (void)tbuf;
-  (void)bars;
   const i64 len_words = rx_div_up(p.len, 32);
   const i64 nwin = rx_div_up(len_words, Bw);
   const i64 w_begin = (i64)seg * p.sw;
   const bool live = w_begin < nwin || seg == 0;
   const i64 w_end = !live ? w_begin : (w_begin + p.sw < nwin ? w_begin + p.sw : nwin);
   Ctx<K> c;
-  rx_ctx_init<G>(p, c, acc, lb);
+  rx_ctx_init<G>(p, c, o, acc, lb);
   u32 pl[8][K];
   u32 xr[K][8];
   u32 *st = sst, *nst = sst + G::NSMAX;
@@ -654,9 +563,6 @@ DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned
   __syncwarp();
   const RxRange ir = rx_interior(p);
   if (w_begin < w_end) rx_fetch<K>(p, ir, c.lane, xr, w_begin * Bw - Lw);
-  // All warps of the CTA run this group; they step through their windows in
-  // lockstep (one barrier per window) so that the SM fetches each line of
-  // the group's straight-line program once for all of them.
   for (int i = 0; i < p.sw; ++i) {
     const i64 w = w_begin + i;
     if (w < w_end) {
@@ -668,13 +574,13 @@ DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned
       if (w + 1 < w_end) rx_fetch<K>(p, ir, c.lane, xr, fword + Bw);  // prefetch the next window
       rx_commit_mask(p, ir, c, Lw, fword);
       if (NS > 0) rx_state_zero(nst, NS, c.lane);
-      G::body(c, pl, st, nst, ~0u);
+      G::body(c, pl, st, nst, rx_all_clusters<G>());
       u32 *t = st;
       st = nst;
       nst = t;
       __syncwarp();
     }
-    if (p.lockstep) __syncthreads();
+    __syncthreads();
   }
   if (!live) return;
   if (NS > 0) {
@@ -686,11 +592,296 @@ DEV void rx_run_segment(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned
   rx_flush<G>(p, c);
 }
 
+// ---------------------------------------------------------------------------
+// Mode choice.  A cluster whose members all have output
+// factors may run output-gated: only in windows whose frame holds one of its
+// output factors, with its incoming state reconstructed on demand.  It pays
+// when the input holds the output factors much more rarely than the first
+// factors -- the prefilter counted both (blocks with a hit per member), so
+// every warp of every kernel of this call makes the same choice.  Returns the
+// mode-B clusters (bit ci).
+// ---------------------------------------------------------------------------
+template <class G> DEV u32 rx_mode_b(const RxParams &p, u32 lane) {
+  if (!p.modeb || !p.pf_on || !p.pf_cnt || G::CBCAP == 0u) return 0u;
+  const u32 *cnt = p.pf_cnt + (u64)G::GID * 64;
+  const u64 nblk = (u64)p.pf_ntiles * 32;
+  const bool mine = lane < (u32)G::NR;
+  const u64 f = mine ? (((G::ALWAYS >> lane) & 1u) ? nblk : (u64)cnt[2 * lane]) : 0ull;
+  const u64 o = mine ? (u64)cnt[2 * lane + 1] : 0ull;
+  u32 bmc = 0u;
+  for (int ci = 0; ci < G::NC; ++ci) {
+    if (!((G::CBCAP >> ci) & 1u)) continue;
+    const u32 cm = G::cmask(ci);
+    const bool in = (cm >> lane) & 1u;
+    u64 F = in ? f : 0ull, O = in ? o : 0ull;
+#pragma unroll
+    for (int s = 16; s > 0; s >>= 1) {
+      F += __shfl_xor_sync(RX_FULL, F, s);
+      O += __shfl_xor_sync(RX_FULL, O, s);
+    }
+    if (6 * O + 16 < F) bmc |= 1u << ci;
+  }
+  return bmc;
+}
+// members of the clusters in `cl`
+template <class G> DEV u32 rx_members_of(u32 cl, u32 lane) {
+  const u32 m = ((int)lane < G::NC && ((cl >> lane) & 1u)) ? G::cmask((int)lane) : 0u;
+  return __reduce_or_sync(RX_FULL, m);
+}
+
+// state words of the clusters in `cl` equal in a and b?
+template <class G> DEV bool rx_state_eq_cl(const u32 *a, const u32 *b, u32 cl, u32 lane) {
+  bool e = true;
+  for (int s = (int)lane; s < G::NS; s += 32)
+    if ((cl >> G::sci(s)) & 1u) e = e && (a[s] == b[s]);
+  return __all_sync(RX_FULL, e);
+}
+
+// Mode-B walk-back: the exact incoming state of window w for the clusters in
+// `stale` (cluster mask).  The group body is monotone in its incoming state
+// (state streams only meet AND / OR / Advance / add-with-carry into a class),
+// so running windows [w-d, w) from the zero state and from the top state
+// (every carry set, every forwarded word all-ones) brackets the true state;
+// once both runs agree, that is the true state.  d doubles until they agree
+// or the walk reaches the stream start (state zero).  Runs are state-only
+// (c.walk: no output) and execute only the stale clusters.
+template <class G>
+DEV void rx_walk_back(const RxParams &p, const RxRange &ir, Ctx<G::K> &c, u32 (&pl)[8][G::K], u32 (&xr)[G::K][8],
+                      i64 w, u32 stale, u32 *st, u32 *wb, i64 len_words) {
+  constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS, M = G::NSMAX;
+  u32 *s0 = wb, *n0 = wb + M, *s1 = wb + 2 * M, *n1 = wb + 3 * M;
+  c.walk = true;
+  int rounds = 0;
+  for (i64 d = 1;; d *= 2) {
+    i64 v0 = w - d;
+    const bool start = v0 <= 0;
+    if (start) v0 = 0;
+    for (int s = (int)c.lane; s < NS; s += 32) {
+      s0[s] = 0u;
+      s1[s] = (!start && ((stale >> G::sci(s)) & 1u)) ? G::top(s) : 0u;
+    }
+    __syncwarp();
+    for (i64 v = v0; v < w; ++v) {
+      const i64 fword = v * Bw - Lw;
+      c.cw = (u32)((len_words - v * Bw) < Bw ? (len_words - v * Bw) : Bw);
+      c.word0 = fword;
+      rx_fetch<K>(p, ir, c.lane, xr, fword);
+      rx_unpack<K>(p, ir, c, xr, pl, fword);
+      rx_commit_mask(p, ir, c, Lw, fword);
+      rx_state_zero(n0, NS, c.lane);
+      G::body(c, pl, s0, n0, stale);
+      u32 *t = s0;
+      s0 = n0;
+      n0 = t;
+      if (!start) {
+        rx_state_zero(n1, NS, c.lane);
+        G::body(c, pl, s1, n1, stale);
+        t = s1;
+        s1 = n1;
+        n1 = t;
+      }
+      __syncwarp();
+    }
+    ++rounds;
+    if (start || rx_state_eq_cl<G>(s0, s1, stale, c.lane)) break;
+  }
+  for (int s = (int)c.lane; s < NS; s += 32)
+    if ((stale >> G::sci(s)) & 1u) st[s] = s0[s];
+  __syncwarp();
+  c.walk = false;
+  if (p.stats && c.lane == 0) {
+    atomicAdd(&p.stats[4], 1ull);
+    atomicAdd(&p.stats[5], (u64)rounds);
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Sparse pass 1 with the prefilter (the default).  Per window the frame's
+// prefilter blocks give the members whose first factor (fm) / output factor
+// (om) occurs there.  Mode-A clusters run where their first factor occurs or
+// state flows in; mode-B clusters run only where their output factor occurs,
+// after rx_walk_back if their state is not known exactly.  Windows where
+// nothing runs are skipped without loading a byte; the bytes of the window
+// expected next are already in flight into a per-warp shared buffer by a TMA
+// bulk copy while the body runs (a wrong guess costs a synchronous load).
+// ---------------------------------------------------------------------------
+#define RX_PF_BLK 1024
+#define RX_PF_TILE 32768
+
+DEV i64 rx_floor_div(i64 a, i64 b) { return a >= 0 ? a / b : -((-a + b - 1) / b); }
+
+template <class G>
+DEV void rx_run_segment_pf(const RxParams &p, int seg, RxOut *o, u64 *acc, u32 *sst, unsigned char *tbuf, u64 *bar,
+                           unsigned char *lb) {
+  constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS, M = G::NSMAX;
+  constexpr u32 WB = 1024u * K;
+  const i64 len_words = rx_div_up(p.len, 32);
+  const i64 nwin = rx_div_up(len_words, Bw);
+  const i64 w_begin = (i64)seg * p.sw;
+  const bool live = w_begin < nwin || seg == 0;
+  const i64 w_end = !live ? w_begin : (w_begin + p.sw < nwin ? w_begin + p.sw : nwin);
+  Ctx<K> c;
+  rx_ctx_init<G>(p, c, o, acc, lb);
+  u32 pl[8][K];
+  u32 xr[K][8];
+  u32 *st = sst, *nst = sst + M, *wbs = sst + 2 * M;
+  const u32 bmc = rx_mode_b<G>(p, c.lane);      // mode-B clusters
+  const u32 bm = rx_members_of<G>(bmc, c.lane);  // ... and their members
+  const u32 always_a = G::ALWAYS & ~bm;
+  for (int s = (int)c.lane; s < NS; s += 32) st[s] = (seg == 0 && p.st_in) ? p.st_in[G::SBASE + s] : 0u;
+  if (c.lane == 0) rx_mbar_init(bar, 1);
+  __syncwarp();
+  const RxRange ir = rx_interior(p);
+  const u32 *gb = p.pf_gbits + (i64)G::GID * p.pf_ntiles;
+  const u32 *mmf = p.pf_mmask + (i64)G::GID * 32 * p.pf_ntiles;
+  const u32 *mmo = p.pf_omask + (i64)G::GID * 32 * p.pf_ntiles;
+  auto frame_blocks = [&](i64 w, i64 &b0, i64 &b1) {
+    i64 flo = (w * Bw - Lw) * 32, fhi = flo + 1024 * K;
+    if (flo < p.avail_lo) flo = p.avail_lo;
+    if (fhi > p.avail_hi) fhi = p.avail_hi;
+    if (fhi <= flo) fhi = flo + 1;
+    b0 = (flo - p.avail_lo) >> 10;
+    b1 = (fhi - 1 - p.avail_lo) >> 10;
+  };
+  i64 bmax = 0;
+  if (w_begin < w_end) {
+    i64 t0;
+    frame_blocks(w_end - 1, t0, bmax);
+  }
+  // a mode-A cluster carries state into the next window
+  auto pending_a = [&](const u32 *a) -> bool {
+    if (NS == 0) return false;
+    return (rx_pend_clusters<G>(a, c.lane) & ~bmc) != 0u;
+  };
+  // first window >= w in which something must run: a block of its frame
+  // holds a first factor of a mode-A member or an output factor of a mode-B
+  // member (w_end if none).  Scans 32 blocks per step, one per lane: groups
+  // whose mode-B members have frequent first factors have a block bit almost
+  // everywhere but need to run rarely.
+  auto next_hit = [&](i64 w) -> i64 {
+    if (w >= w_end) return w_end;
+    if (always_a != 0u) return w;
+    i64 b0, b1;
+    frame_blocks(w, b0, b1);
+    for (i64 c0 = b0 & ~(i64)31; c0 <= bmax; c0 += 32) {
+      const u32 word = gb[c0 >> 5];
+      const i64 b = c0 + c.lane;
+      bool need = false;
+      if (((word >> c.lane) & 1u) && b >= b0 && b <= bmax) need = ((mmf[b] & ~bm) | (mmo[b] & bm)) != 0u;
+      const u32 bal = __ballot_sync(RX_FULL, need);
+      if (!bal) continue;
+      const i64 bb = c0 + (__ffs(bal) - 1);
+      if (bb <= b1) return w;
+      const i64 pos = p.avail_lo + bb * RX_PF_BLK;
+      const i64 wn = rx_floor_div(rx_floor_div(pos, 32) + Lw - 32 * K, Bw) + 1;
+      const i64 r = wn > w + 1 ? wn : w + 1;
+      return r < w_end ? r : w_end;
+    }
+    return w_end;
+  };
+  i64 staged = -1;  // window whose bytes are in flight / in tbuf (-1: none)
+  u32 phase = 0;
+  auto stage = [&](i64 w) {
+    const i64 f = w * Bw - Lw;
+    if (w < w_end && f >= ir.lo && f + 32 * K <= ir.hi) {
+      __syncwarp();
+      if (c.lane == 0) rx_bulk_load(tbuf, p.in + f * 32, WB, bar);
+      staged = w;
+    }
+  };
+  auto retire = [&]() {  // wait for the copy in flight (keeps the mbarrier phase in step)
+    rx_mbar_wait(bar, phase);
+    phase ^= 1u;
+    staged = -1;
+  };
+  u32 exact = 0u;  // mode-B clusters whose state in st[] is exact at window w
+  i64 w = pending_a(st) ? w_begin : next_hit(w_begin);
+  if (w < w_end) stage(w);
+  while (w < w_end) {
+    const u32 pendc = NS > 0 ? rx_pend_clusters<G>(st, c.lane) : 0u;
+    const bool pend_in = (pendc & ~bmc) != 0u;
+    if (p.stats && c.lane == 0) atomicAdd(&p.stats[3], 1ull);
+    i64 b0, b1;
+    frame_blocks(w, b0, b1);
+    u32 fmine = 0u, omine = 0u;
+    for (i64 b = b0 + c.lane; b <= b1; b += 32)
+      if ((gb[b >> 5] >> (b & 31)) & 1u) {
+        fmine |= mmf[b];
+        omine |= mmo[b];
+      }
+    const u32 fm = __reduce_or_sync(RX_FULL, fmine), om = __reduce_or_sync(RX_FULL, omine);
+    const u32 rmask = (fm & ~bm) | (om & bm);
+    if (rmask == 0u && !pend_in && always_a == 0u) {
+      exact = 0u;
+      w = next_hit(w + 1);
+      continue;
+    }
+    // the clusters to run; those of them in mode B whose state is stale
+    // first reconstruct it
+    const u32 run = rx_run_clusters<G>(rmask, bmc, pendc, c.lane);
+    const u32 runb = run & bmc;
+    const u32 stale = runb & ~exact;
+    if (stale) rx_walk_back<G>(p, ir, c, pl, xr, w, stale, st, wbs, len_words);
+    const i64 fword = w * Bw - Lw;
+    if (staged == w) {
+      retire();
+      const uint4 *q = reinterpret_cast<const uint4 *>(tbuf + c.lane * (32u * K));
+#pragma unroll
+      for (int k = 0; k < K; ++k) {
+        const uint4 a0 = q[2 * k], a1 = q[2 * k + 1];
+        xr[k][0] = a0.x; xr[k][1] = a0.y; xr[k][2] = a0.z; xr[k][3] = a0.w;
+        xr[k][4] = a1.x; xr[k][5] = a1.y; xr[k][6] = a1.z; xr[k][7] = a1.w;
+      }
+    } else {
+      if (staged >= 0) retire();  // a stale guess: drain it
+      rx_fetch<K>(p, ir, c.lane, xr, fword);
+    }
+    // guess the next window and start its copy before the body runs
+    if (staged < 0) stage(pend_in ? w + 1 : next_hit(w + 1));
+    if (p.stats && c.lane == 0) {
+      atomicAdd(&p.stats[0], 1ull);
+      atomicAdd(&p.stats[2], (u64)__popc(rmask));
+      atomicAdd(&p.stats[6], (u64)__popc(run));
+      u64 *gs = p.stats + 8 + 4 * G::GID;  // per group: active windows, member hits, mode-B clusters, cluster runs
+      atomicAdd(&gs[0], 1ull);
+      atomicAdd(&gs[1], (u64)__popc(rmask));
+      gs[2] = (u64)__popc(bmc);
+      atomicAdd(&gs[3], (u64)__popc(run));
+    }
+    c.cw = (u32)((len_words - w * Bw) < Bw ? (len_words - w * Bw) : Bw);
+    c.word0 = fword;
+    rx_unpack<K>(p, ir, c, xr, pl, fword);
+    rx_commit_mask(p, ir, c, Lw, fword);
+    if (NS > 0) rx_state_zero(nst, NS, c.lane);
+    G::body_i(c, pl, st, nst, run);
+    u32 *t = st;
+    st = nst;
+    nst = t;
+    __syncwarp();
+    exact = runb;  // the mode-B clusters that ran now hold their exact end state
+    const i64 nw = pending_a(st) ? w + 1 : next_hit(w + 1);
+    if (nw != w + 1) exact = 0u;
+    w = nw;
+  }
+  if (staged >= 0) retire();
+  if (!live) return;
+  if (NS > 0) {
+    // mode-B slots are not carried across segments (the next segment walks
+    // back for itself): the fix-up sees zero for them on both sides
+    u32 *dst = p.seg_state + ((i64)seg * G::NG + G::GID) * G::NSMAX;
+    for (int s = (int)c.lane; s < NS; s += 32) dst[s] = ((bmc >> G::sci(s)) & 1u) ? 0u : st[s];
+    if (p.st_out && w_end == nwin)
+      for (int s = (int)c.lane; s < NS; s += 32) p.st_out[G::SBASE + s] = st[s];
+  }
+  rx_flush<G>(p, c);
+}
+
 // Fix-up / rematch (one warp per group): walk the windows in order carrying
 // the true state; wherever it differs from the state pass 1 used, re-run the
-// window with both states and apply (new - old) until they agree.
+// window with both states and apply (new - old) until they agree.  Mode-B
+// clusters (exact in pass 1 already) do not run here.
 template <class G>
-DEV void rx_fixup_group(const RxParams &p, u64 *acc, u32 *sst, unsigned char *lb, int fseg) {
+DEV void rx_fixup_group(const RxParams &p, RxOut *o, u64 *acc, u32 *sst, unsigned char *lb, int fseg) {
   constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS, M = G::NSMAX;
   if (NS == 0) return;
   const i64 len_words = rx_div_up(p.len, 32);
@@ -699,12 +890,15 @@ DEV void rx_fixup_group(const RxParams &p, u64 *acc, u32 *sst, unsigned char *lb
   if (p.fix_phase == 1 && (fseg <= 0 || fseg >= nseg)) return;
   auto sstate = [&](const u32 *base, i64 seg) { return base + (seg * G::NG + G::GID) * G::NSMAX; };
   Ctx<K> c;
-  rx_ctx_init<G>(p, c, acc, lb);
+  rx_ctx_init<G>(p, c, o, acc, lb);
+  // mode-B clusters were exact in pass 1 already: only the others re-run
+  const u32 runa = rx_all_clusters<G>() & ~(p.mode == 1 ? rx_mode_b<G>(p, c.lane) : 0u);
   u32 pl[8][K];
   u32 xr[K][8];
   u32 *tru = sst, *old = sst + M, *t1 = sst + 2 * M, *t2 = sst + 3 * M;
   u32 fold[G::NR * K];
-  c.fold = p.match_total ? fold : nullptr;
+  if (c.lane == 0) o->fold = p.match_total ? fold : nullptr;
+  __syncwarp();
   // re-run windows [w0, w1) with both states (old: the state the applied
   // results assumed, subtracted; tru: the true state, added) until the two
   // runs' states agree; returns whether they did
@@ -720,17 +914,25 @@ DEV void rx_fixup_group(const RxParams &p, u64 *acc, u32 *sst, unsigned char *lb
       rx_unpack<K>(p, ir, c, xr, pl, fword);
       rx_commit_mask(p, ir, c, Lw, fword);
       // old run: subtract
-      c.sign = ~0ull;
-      c.want_dense = false;
-      if (c.fold)
+      if (c.lane == 0) {
+        o->sign = ~0ull;
+        o->want_dense = 0;
+      }
+      c.dense = false;
+      if (p.match_total)  // each lane's own copy (local memory)
         for (int j = 0; j < G::NR * K; ++j) fold[j] = 0u;
+      __syncwarp();
       rx_state_zero(t1, NS, c.lane);
-      G::body(c, pl, old, t1, ~0u);
+      G::body(c, pl, old, t1, runa);
       // new run: add, rewrite dense words
-      c.sign = 1ull;
-      c.want_dense = p.dense != nullptr;
+      if (c.lane == 0) {
+        o->sign = 1ull;
+        o->want_dense = p.dense != nullptr;
+      }
+      c.dense = p.dense != nullptr;
+      __syncwarp();
       rx_state_zero(t2, NS, c.lane);
-      G::body(c, pl, tru, t2, ~0u);
+      G::body(c, pl, tru, t2, runa);
       __syncwarp();
       rx_state_copy(old, t1, NS, c.lane);
       rx_state_copy(tru, t2, NS, c.lane);
@@ -789,48 +991,32 @@ DEV void rx_fixup_group(const RxParams &p, u64 *acc, u32 *sst, unsigned char *lb
     rx_flush<G>(p, c);
     return;
   }
-  // serial form (rematch, mode 2; and mode 1 with fix_phase 0): one warp
-  // walks the segments in order carrying the true state
+  // serial form (rematch, mode 2): one warp walks the chunk carrying the true
+  // state from the caller's assumed one until they agree
   for (int s = (int)c.lane; s < NS; s += 32) {
     tru[s] = p.st_in ? p.st_in[G::SBASE + s] : 0u;
-    old[s] = (p.mode == 2 && p.st_assumed) ? p.st_assumed[G::SBASE + s] : 0u;
+    old[s] = p.st_assumed ? p.st_assumed[G::SBASE + s] : 0u;
   }
   __syncwarp();
-  for (i64 seg = 0; seg < nseg; ++seg) {
-    const i64 w_begin = seg * p.sw;
-    const i64 w_end = w_begin + p.sw < nwin ? w_begin + p.sw : nwin;
-    if (p.mode == 1) {
-      // the state pass 1 assumed for this segment
-      for (int s = (int)c.lane; s < NS; s += 32) old[s] = seg == 0 ? (p.st_in ? p.st_in[G::SBASE + s] : 0u) : 0u;
-      __syncwarp();
-    }
-    const bool conv = walk(w_begin, w_end);
-    if (conv) {
-      if (p.mode == 2) break;  // identical to the caller's run from here on
-      // from here on pass 1's result stands: take its segment end state
-      const u32 *src = sstate(p.seg_state, seg);
-      for (int s = (int)c.lane; s < NS; s += 32) tru[s] = src[s];
-      __syncwarp();
-    }
-    if (seg == nseg - 1 && p.st_out && (p.mode == 1 || !conv))
-      for (int s = (int)c.lane; s < NS; s += 32) p.st_out[G::SBASE + s] = tru[s];
-  }
+  const bool conv = walk(0, nwin);
+  if (p.st_out && !conv)
+    for (int s = (int)c.lane; s < NS; s += 32) p.st_out[G::SBASE + s] = tru[s];
   rx_flush<G>(p, c);
 }
 
 // ---------------------------------------------------------------------------
 // Cross-regex prefilter.
-// One streaming pass over the input: for every position q the 4 bytes ending
-// at q form x (little-endian, byte q on top); its last two bytes index a
-// 65,536-bit bigram bitmap held in shared memory; on a hit the (few) factor
-// grams ending in that bigram are verified exactly against x.  A tile of 32
-// blocks of 1 KiB is owned by one CTA, which records per block the factor
-// ids found (deduplicated, up to 15) and per group a 32-bit word with one bit
-// per block in which one of the group's factors occurs.
+// One streaming pass over the input.  For every position q, x = the 4 bytes
+// ending at q (little-endian, byte q on top) is tested against the anchor
+// filters held in shared memory (a Bloom filter over the 4-gram anchors and,
+// if the program has any, one over the 3-gram anchors and a bitmap over the
+// 2-gram anchors).  Filter hits are compacted per warp and verified one per
+// lane: the anchor's hash chain, then each factor's 16-byte extension window
+// around q.  A tile of 32 blocks of 1 KiB is owned by one CTA, which ORs the
+// member masks of the factors found into shared per-(group, block) masks
+// (first / output factors apart), then writes per group one word of block
+// bits, the masks of the blocks hit, and per-member block counts.
 // ---------------------------------------------------------------------------
-#define RX_PF_BLK 1024
-#define RX_PF_TILE 32768
-
 DEV u32 rx_load_u32_slow(const RxParams &p, i64 pos) {
   u32 v = 0u;
   for (int j = 0; j < 4; ++j) {
@@ -840,77 +1026,104 @@ DEV u32 rx_load_u32_slow(const RxParams &p, i64 pos) {
   return v;
 }
 
-// x of position base + r (0 <= r < 20; 4 bytes ending there) from the words w0 (bytes base-4..base-1) .. w5 (base+16..base+19)
-DEV u32 rx_pf_x(u32 w0, u32 w1, u32 w2, u32 w3, u32 w4, u32 w5, int r) {
+// 4 bytes ending at position base + r (0 <= r < 16) from the words w0 (bytes
+// base-4..base-1) .. w4 (base+12..base+15)
+DEV u32 rx_pf_x(u32 w0, u32 w1, u32 w2, u32 w3, u32 w4, int r) {
   const int m = r >> 2, s = r & 3;
-  const u32 lo = m == 0 ? w0 : (m == 1 ? w1 : (m == 2 ? w2 : (m == 3 ? w3 : w4)));
-  const u32 hi = m == 0 ? w1 : (m == 1 ? w2 : (m == 2 ? w3 : (m == 3 ? w4 : w5)));
+  const u32 lo = m == 0 ? w0 : (m == 1 ? w1 : (m == 2 ? w2 : w3));
+  const u32 hi = m == 0 ? w1 : (m == 1 ? w2 : (m == 2 ? w3 : w4));
   return s == 3 ? hi : __funnelshift_r(lo, hi, 8 * (s + 1));
 }
 
-// One queued hit of an index bigram: its end position (offset in the tile),
-// the 4 bytes ending there (xa) and the 4 bytes after them (xc); the gram
-// ends d = 0..3 bytes later and is x(d) = funnel(xa, xc, 8d).  It is recorded
-// in the block of the bigram's end (inside the gram, hence inside every
-// window frame that contains the gram): the (group, member mask) pairs of the
-// factor are ORed into the tile's shared per-(group, block) member masks.
-DEV void rx_pf_record(const RxParams &p, const u32 *T, u32 *sm, u32 fid, int b) {
-  const u32 f1 = T[p.pf_o_fgoff + fid + 1];
-  for (u32 j = T[p.pf_o_fgoff + fid]; j < f1; ++j) {
-    u32 *a = &sm[T[p.pf_o_fgent + 2 * j] * 32u + (u32)b];
-    const u32 m = T[p.pf_o_fgent + 2 * j + 1];
-    if ((*(volatile u32 *)a & m) != m) atomicOr(a, m);
+// the 16-byte extension window of factor entry E ({ae, v[4], m[4], ...})
+// for an anchor ending at q
+DEV bool rx_pf_ext_ok(const RxParams &p, const u32 *E, i64 q) {
+  const i64 s = q - (i64)E[0];
+  u32 w[4];
+  if (s - 3 >= p.avail_lo && s + 20 <= p.avail_hi) {
+    const unsigned long long ad = (unsigned long long)(p.in + s);
+    const u32 *al = reinterpret_cast<const u32 *>(ad & ~3ull);
+    const u32 sh = (u32)(ad & 3ull) * 8u;
+    const u32 x0 = __ldg(al), x1 = __ldg(al + 1), x2 = __ldg(al + 2), x3 = __ldg(al + 3), x4 = __ldg(al + 4);
+    w[0] = __funnelshift_r(x0, x1, sh);
+    w[1] = __funnelshift_r(x1, x2, sh);
+    w[2] = __funnelshift_r(x2, x3, sh);
+    w[3] = __funnelshift_r(x3, x4, sh);
+  } else {
+    // near the readable range's ends: a byte outside it never matches a
+    // compared (masked) position
+    for (int j = 0; j < 4; ++j) {
+      u32 v = 0u, out = 0u;
+      for (int b = 0; b < 4; ++b) {
+        const i64 ps = s + 4 * j + b;
+        if (ps >= p.avail_lo && ps < p.avail_hi) v |= (u32)p.in[ps] << (8 * b);
+        else out |= 0xffu << (8 * b);
+      }
+      if (out & E[5 + j]) return false;
+      w[j] = v;
+    }
   }
+  return ((w[0] & E[5]) == E[1]) && ((w[1] & E[6]) == E[2]) && ((w[2] & E[7]) == E[3]) && ((w[3] & E[8]) == E[4]);
 }
 
-DEV void rx_pf_hit(const RxParams &p, const u32 *T, u32 *sm, u32 off, u32 xa, u32 xc, i64 tile_lo) {
-  const u32 bg = xa >> 16, wi = bg >> 5, bit = bg & 31u;
-  const u32 idx = T[2048 + wi] + __popc(T[wi] & ((1u << bit) - 1u));
-  u32 shapes = T[4096 + idx];
-  const int b = (int)(off >> 10);
-  const i64 q0 = tile_lo + off;
+DEV u32 rx_pf_ht_hash(u32 gram, u32 k) { return (gram ^ (k * 0x27D4EB2Fu)) * 0x9E3779B1u; }
+
+// verify one filter hit: x = the 4 bytes ending at q, kbits: bit k-2 set if
+// the k-gram filter fired
+DEV void rx_pf_verify(const RxParams &p, u32 *sm, int NG, u32 x, u32 kbits, i64 q, int b) {
+  const u32 *T = p.pf_tab;
   const u32 hmask = (1u << p.pf_hbits) - 1u;
-  const u32 *H = T + p.pf_o_ent;
-  while (shapes) {
-    const u32 sh = __ffs(shapes) - 1;
-    shapes &= shapes - 1u;
-    const u32 k = sh / 3u + 2u, d = sh - 3u * (k - 2u);
-    const u32 mask = k == 4u ? 0xffffffffu : (0xffffffffu << (8u * (4u - k)));
-    const u32 key = (d == 0u ? xa : __funnelshift_r(xa, xc, 8u * d)) & mask;
-    const i64 q = q0 + d;
-    if (q >= p.avail_hi || q - (i64)k + 1 < p.avail_lo) continue;
-    u32 h = ((key ^ (sh * 0x85EBCA6Bu)) * 0x9E3779B1u) >> (32u - p.pf_hbits);
+  for (u32 k = 4; k >= 2; --k) {
+    if (!((kbits >> (k - 2)) & 1u)) continue;
+    const u32 gmask = k == 4 ? 0xffffffffu : (0xffffffffu << (8u * (4u - k)));
+    const u32 gram = x & gmask;
+    if (q - (i64)k + 1 < p.avail_lo) continue;
+    u32 h = rx_pf_ht_hash(gram, k) >> (32u - p.pf_hbits);
     for (;;) {
-      const u32 tag = H[2 * h + 1];
-      if (tag == 0u) break;
-      if (H[2 * h] == key && ((tag >> 1) & 127u) == sh) rx_pf_record(p, T, sm, tag >> 8, b);
+      const uint4 e = __ldg(reinterpret_cast<const uint4 *>(T + p.pf_o_ht) + h);
+      if (e.y == 0u) break;
+      if (e.x == gram && e.y == ((k << 1) | 1u)) {
+        for (u32 j = 0; j < e.w; ++j) {
+          const u32 *E = T + p.pf_o_ext + 12u * (e.z + j);
+          if (!rx_pf_ext_ok(p, E, q)) continue;
+          const u32 t0 = __ldg(&E[9]), tn = __ldg(&E[10]);
+          for (u32 t = t0; t < t0 + tn; ++t) {
+            const u32 g = __ldg(&T[p.pf_o_fgent + 3 * t]), m = __ldg(&T[p.pf_o_fgent + 3 * t + 1]),
+                      kind = __ldg(&T[p.pf_o_fgent + 3 * t + 2]);
+            u32 *a = &sm[(kind * (u32)NG + g) * 32u + (u32)b];
+            if ((*(volatile u32 *)a & m) != m) atomicOr(a, m);
+          }
+        }
+      }
       h = (h + 1u) & hmask;
     }
   }
 }
 
-// smem: [tables (if they fit) | member masks NG x 32 | per-warp hit queues 32 x 3]
-DEV void rx_prefilter_run(const RxParams &p, int NG, bool tab_in_smem) {
+// smem: [filters (pf_smem_words) | member masks 2 x NG x 32 | per-warp hit queues 32 x 3]
+DEV void rx_prefilter_run(const RxParams &p, int NG) {
   extern __shared__ __align__(16) u32 pf_smem[];
   const int tid = threadIdx.x, nt = blockDim.x;
-  const u32 tw = tab_in_smem ? ((p.pf_words + 3u) & ~3u) : 4096u;
+  const u32 tw = (p.pf_smem_words + 3u) & ~3u;
   u32 *tab = pf_smem;
-  for (u32 i = tid; i < tw && i < p.pf_words; i += nt) tab[i] = __ldg(&p.pf_tab[i]);
-  // l1 + rank are always staged; the rest is read through T
-  const u32 *T = tab_in_smem ? (const u32 *)tab : p.pf_tab;
-  u32 *sm = pf_smem + tw;                     // [NG][32 blocks] member masks
-  u32 *wq = sm + 32 * NG + 96 * (tid >> 5);  // per-warp hit queue: 32 x {off, xa, xc}
+  for (u32 i = tid; i < p.pf_smem_words; i += nt) tab[i] = __ldg(&p.pf_tab[i]);
+  u32 *sm = pf_smem + tw;                      // [2][NG][32 blocks] member masks
+  u32 *wq = sm + 64 * NG + 96 * (tid >> 5);   // per-warp hit queue: 32 x {offset, x, kbits}
+  const u32 *bl4 = tab, *bl3 = tab + p.pf_o_b3, *bg2 = tab + p.pf_o_b2;
+  const bool has3 = p.pf_o_b3 != 0u, has2 = p.pf_o_b2 != 0u;
+  const u32 s4 = 32u - p.pf_b4bits, s3 = 32u - p.pf_b3bits;
   const u32 lane = rx_lane();
   const i64 span = p.avail_hi - p.avail_lo;
   const i64 ntiles = (span + RX_PF_TILE - 1) / RX_PF_TILE;
+  const i64 nblk = 32 * p.pf_ntiles;
   for (i64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
-    for (int i = tid; i < 32 * NG; i += nt) sm[i] = 0u;
+    for (int i = tid; i < 64 * NG; i += nt) sm[i] = 0u;
     __syncthreads();
     const i64 tile_lo = p.avail_lo + t * RX_PF_TILE;
     for (int j = 0; j < RX_PF_TILE / 16; j += nt) {
       const i64 base = tile_lo + (i64)(j + tid) * 16;
       u32 w1, w2, w3, w4;
-      if (p.pf_aligned && base + 16 <= p.avail_hi) {
+      if (p.aligned && ((p.avail_lo & 15) == 0) && base + 16 <= p.avail_hi) {
         const uint4 v = __ldg(reinterpret_cast<const uint4 *>(p.in + base));
         w1 = v.x; w2 = v.y; w3 = v.z; w4 = v.w;
       } else {
@@ -920,21 +1133,30 @@ DEV void rx_prefilter_run(const RxParams &p, int NG, bool tab_in_smem) {
         w4 = rx_load_u32_slow(p, base + 12);
       }
       u32 w0 = __shfl_up_sync(RX_FULL, w4, 1);
-      if (lane == 0) w0 = rx_load_u32_slow(p, base - 4);
-      u32 w5 = __shfl_down_sync(RX_FULL, w1, 1);
-      if (lane == 31) w5 = rx_load_u32_slow(p, base + 16);
-      // pass 1: bigram bitmap test of the 16 positions -> hit mask
-      u32 hm = 0u;
+      if (lane == 0)
+        w0 = (p.aligned && ((p.avail_lo & 15) == 0) && base - 4 >= p.avail_lo && base <= p.avail_hi)
+                 ? __ldg(reinterpret_cast<const u32 *>(p.in + base - 4))
+                 : rx_load_u32_slow(p, base - 4);
+      // filter pass over the 16 positions -> hit masks per anchor length
+      u32 h4 = 0u, h3 = 0u, h2 = 0u;
 #pragma unroll
       for (int r = 0; r < 16; ++r) {
-        const u32 x = rx_pf_x(w0, w1, w2, w3, w4, w5, r);
-        const u32 bg = x >> 16;
-        hm |= ((tab[bg >> 5] >> (bg & 31)) & 1u) << r;
+        const u32 x = rx_pf_x(w0, w1, w2, w3, w4, r);
+        const u32 a = (x * 0x9E3779B1u) >> s4;
+        h4 |= ((bl4[a >> 5] >> (a & 31u)) & 1u) << r;
+        if (has3) {
+          const u32 b = ((x >> 8) * 0x85EBCA77u) >> s3;
+          h3 |= ((bl3[b >> 5] >> (b & 31u)) & 1u) << r;
+        }
+        if (has2) {
+          const u32 g = x >> 16;
+          h2 |= ((bg2[g >> 5] >> (g & 31u)) & 1u) << r;
+        }
       }
+      u32 hm = h4 | h3 | h2;
       const i64 rem = p.avail_hi - base;
       if (rem < 16) hm &= rem <= 0 ? 0u : ((1u << rem) - 1u);
-      // pass 2: the warp's hits are compacted into a queue of 32 and checked
-      // one per lane (exact gram compare)
+      // the warp's hits are compacted into a queue of 32 and verified one per lane
       u32 qn = 0;
       for (;;) {
         const u32 bal = __ballot_sync(RX_FULL, hm != 0u);
@@ -945,14 +1167,17 @@ DEV void rx_prefilter_run(const RxParams &p, int NG, bool tab_in_smem) {
             hm &= hm - 1u;
             u32 *e = wq + 3 * (qn + rk);
             e[0] = (u32)(base + r - tile_lo);
-            e[1] = rx_pf_x(w0, w1, w2, w3, w4, w5, r);
-            e[2] = rx_pf_x(w0, w1, w2, w3, w4, w5, r + 4);
+            e[1] = rx_pf_x(w0, w1, w2, w3, w4, r);
+            e[2] = ((h4 >> r) & 1u) << 2 | ((h3 >> r) & 1u) << 1 | ((h2 >> r) & 1u);
           }
           qn = qn + __popc(bal) < 32u ? qn + __popc(bal) : 32u;
         }
         if (qn == 32u || (bal == 0u && qn > 0u)) {
           __syncwarp();
-          if (lane < qn) rx_pf_hit(p, T, sm, wq[3 * lane], wq[3 * lane + 1], wq[3 * lane + 2], tile_lo);
+          if (lane < qn) {
+            const u32 off = wq[3 * lane];
+            rx_pf_verify(p, sm, NG, wq[3 * lane + 1], wq[3 * lane + 2], tile_lo + off, (int)(off >> 10));
+          }
           __syncwarp();
           qn = 0;
         }
@@ -960,440 +1185,26 @@ DEV void rx_prefilter_run(const RxParams &p, int NG, bool tab_in_smem) {
       }
     }
     __syncthreads();
-    // one warp per group: lane b holds block b's member mask; the group's
-    // tile word of block bits is their ballot
-    const i64 nblk = 32 * p.pf_ntiles;
+    // one warp per group: lane b holds block b's member masks; the group's
+    // tile word of block bits is their ballot; lane m counts member m's blocks
     for (int g = tid >> 5; g < NG; g += nt >> 5) {
-      const u32 v = sm[32 * g + lane];
-      const u32 bal = __ballot_sync(RX_FULL, v != 0u);
+      const u32 f = sm[32 * g + lane], o = sm[32 * (NG + g) + lane];
+      const u32 bal = __ballot_sync(RX_FULL, (f | o) != 0u);
       if (lane == 0) p.pf_gbits[(i64)g * p.pf_ntiles + t] = bal;
-      if (v) p.pf_mmask[(i64)g * nblk + t * 32 + lane] = v;
+      if (f | o) {
+        p.pf_mmask[(i64)g * nblk + t * 32 + lane] = f;
+        p.pf_omask[(i64)g * nblk + t * 32 + lane] = o;
+      }
+      if (bal && p.pf_cnt) {
+        u32 cf = 0u, co = 0u;
+        for (int b = 0; b < 32; ++b) {
+          cf += (__shfl_sync(RX_FULL, f, b) >> lane) & 1u;
+          co += (__shfl_sync(RX_FULL, o, b) >> lane) & 1u;
+        }
+        if (cf) atomicAdd(&p.pf_cnt[(g * 32 + lane) * 2], cf);
+        if (co) atomicAdd(&p.pf_cnt[(g * 32 + lane) * 2 + 1], co);
+      }
     }
     __syncthreads();
   }
-}
-
-// first block >= b0 (and <= bmax) whose bit is set in the group's bitmap;
-// returns bmax + 1 if none (warp-uniform)
-DEV i64 rx_pf_next(const u32 *gb, i64 b0, i64 bmax, u32 lane) {
-  for (i64 w0 = b0 >> 5; w0 <= (bmax >> 5); w0 += 32) {
-    const i64 wi = w0 + lane;
-    u32 v = wi <= (bmax >> 5) ? gb[wi] : 0u;
-    if (wi == (b0 >> 5)) v &= RX_FULL << (b0 & 31);
-    const u32 bal = __ballot_sync(RX_FULL, v != 0u);
-    if (bal) {
-      const int l = __ffs(bal) - 1;
-      const u32 vv = __shfl_sync(RX_FULL, v, l);
-      const i64 b = (w0 + l) * 32 + (__ffs(vv) - 1);
-      return b <= bmax ? b : bmax + 1;
-    }
-  }
-  return bmax + 1;
-}
-
-DEV i64 rx_floor_div(i64 a, i64 b) { return a >= 0 ? a / b : -((-a + b - 1) / b); }
-
-// Pass 1 with the prefilter: windows whose frame holds no factor of the group
-// and into which no state flows are skipped without loading a byte; the
-// others run only the members whose factor occurs in the frame, that carry
-// state, or that have no factor (G::ALWAYS).
-template <class G> DEV void rx_run_segment_pf(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *lb) {
-  constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS;
-  const i64 len_words = rx_div_up(p.len, 32);
-  const i64 nwin = rx_div_up(len_words, Bw);
-  const i64 w_begin = (i64)seg * p.sw;
-  const bool live = w_begin < nwin || seg == 0;
-  const i64 w_end = !live ? w_begin : (w_begin + p.sw < nwin ? w_begin + p.sw : nwin);
-  Ctx<K> c;
-  rx_ctx_init<G>(p, c, acc, lb);
-  u32 pl[8][K];
-  u32 xr[K][8];
-  u32 *st = sst, *nst = sst + G::NSMAX;
-  for (int s = (int)c.lane; s < NS; s += 32) st[s] = (seg == 0 && p.st_in) ? p.st_in[G::SBASE + s] : 0u;
-  __syncwarp();
-  const RxRange ir = rx_interior(p);
-  const u32 *gb = p.pf_gbits + (i64)G::GID * p.pf_ntiles;
-  auto frame_blocks = [&](i64 w, i64 &b0, i64 &b1) {
-    i64 flo = (w * Bw - Lw) * 32, fhi = flo + 1024 * K;
-    if (flo < p.avail_lo) flo = p.avail_lo;
-    if (fhi > p.avail_hi) fhi = p.avail_hi;
-    if (fhi <= flo) fhi = flo + 1;
-    b0 = (flo - p.avail_lo) >> 10;
-    b1 = (fhi - 1 - p.avail_lo) >> 10;
-  };
-  i64 bmax = 0;
-  if (w_begin < w_end) {
-    i64 t0;
-    frame_blocks(w_end - 1, t0, bmax);
-  }
-  // lockstep (p.lockstep): the CTA's warps step through window i together
-  // (one barrier per step) so that they fetch the group's code together;
-  // otherwise each warp jumps to its next window with a factor hit
-  const bool lockstep = p.lockstep != 0;
-  i64 w = w_begin;
-  int step = 0;
-  while (lockstep ? step < p.sw : w < w_end) {
-    if (lockstep) {
-      if (step > 0) __syncthreads();
-      w = w_begin + step;
-      ++step;
-      if (w >= w_end) continue;
-    }
-    i64 b0, b1;
-    frame_blocks(w, b0, b1);
-    bool pend = false;
-    if (NS > 0) {
-      bool any = false;
-      for (int s = (int)c.lane; s < NS; s += 32) any = any || st[s] != 0u;
-      pend = __any_sync(RX_FULL, any);
-    }
-    if (p.stats && c.lane == 0) atomicAdd(&p.stats[3], 1ull);  // [3] window visits (checks)
-    if (p.dbg == 1) {
-      if (lockstep) continue;
-      ++w;
-      continue;
-    }
-    if (!pend && G::ALWAYS == 0u) {
-      const i64 b = rx_pf_next(gb, b0, lockstep ? b1 : bmax, c.lane);
-      if (lockstep && b > b1) continue;
-      if (b > b1) {
-        if (b > bmax) break;
-        // the first window whose frame reaches block b
-        const i64 pos = p.avail_lo + b * RX_PF_BLK;
-        const i64 wn = rx_floor_div(rx_floor_div(pos, 32) + Lw - 32 * K, Bw) + 1;
-        w = wn > w + 1 ? wn : w + 1;
-        continue;
-      }
-    }
-    // members whose factor occurs in one of the frame's blocks (lane i
-    // looks at block b0 + i; a frame spans a few blocks)
-    const u32 *mm = p.pf_mmask + (i64)G::GID * 32 * p.pf_ntiles;
-    u32 mine = 0u;
-    for (i64 b = b0 + c.lane; b <= b1; b += 32)
-      if ((gb[b >> 5] >> (b & 31)) & 1u) mine |= mm[b];
-    const u32 rmask = __reduce_or_sync(RX_FULL, mine);
-    if (p.stats && c.lane == 0) {
-      // [0] active windows [1] of them only for carried state [2] members hit
-      atomicAdd(&p.stats[0], 1ull);
-      if (rmask == 0u) atomicAdd(&p.stats[1], 1ull);
-      atomicAdd(&p.stats[2], (u64)__popc(rmask));
-    }
-    const i64 cstart = w * Bw;
-    const i64 fword = cstart - Lw;
-    c.cw = (u32)((len_words - cstart) < Bw ? (len_words - cstart) : Bw);
-    c.word0 = fword;
-    rx_fetch<K>(p, ir, c.lane, xr, fword);
-    rx_unpack<K>(p, ir, c, xr, pl, fword);
-    rx_commit_mask(p, ir, c, Lw, fword);
-    if (NS > 0) rx_state_zero(nst, NS, c.lane);
-    if (p.dbg == 2) {
-      if (c.lane == 0 && (pl[0][0] ^ pl[7][K - 1]) == 0x12345u) atomicAdd(p.status, 0u);  // keep the loads
-    } else {
-      G::body(c, pl, st, nst, rmask);
-    }
-    u32 *t = st;
-    st = nst;
-    nst = t;
-    __syncwarp();
-    if (!lockstep) ++w;
-  }
-  if (lockstep && step > 0) __syncthreads();
-  if (!live) return;
-  if (NS > 0) {
-    u32 *dst = p.seg_state + ((i64)seg * G::NG + G::GID) * G::NSMAX;
-    for (int s = (int)c.lane; s < NS; s += 32) dst[s] = st[s];
-    if (p.st_out && w_end == nwin)
-      for (int s = (int)c.lane; s < NS; s += 32) p.st_out[G::SBASE + s] = st[s];
-  }
-  rx_flush<G>(p, c);
-}
-
-// Sparse pass 1 with a one-window lookahead (the default): while the body
-// of window w runs, the bytes of the window expected next -- w + 1 if state
-// flows into w (it usually flows on), else the next window whose frame holds
-// a factor of the group -- are already on their way into a per-warp shared
-// buffer by a TMA bulk copy.  A wrong guess costs a synchronous global load;
-// the window order and the set of windows run are exactly those of
-// rx_run_segment_pf (running an extra window with no state and no factor is
-// harmless: its output and state are zero).
-template <class G>
-DEV void rx_run_segment_pf_staged(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *tbuf, u64 *bar,
-                                  unsigned char *lb) {
-  constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS;
-  constexpr u32 WB = 1024u * K;
-  const i64 len_words = rx_div_up(p.len, 32);
-  const i64 nwin = rx_div_up(len_words, Bw);
-  const i64 w_begin = (i64)seg * p.sw;
-  const bool live = w_begin < nwin || seg == 0;
-  const i64 w_end = !live ? w_begin : (w_begin + p.sw < nwin ? w_begin + p.sw : nwin);
-  Ctx<K> c;
-  rx_ctx_init<G>(p, c, acc, lb);
-  u32 pl[8][K];
-  u32 xr[K][8];
-  u32 *st = sst, *nst = sst + G::NSMAX;
-  for (int s = (int)c.lane; s < NS; s += 32) st[s] = (seg == 0 && p.st_in) ? p.st_in[G::SBASE + s] : 0u;
-  if (c.lane == 0) rx_mbar_init(bar, 1);
-  __syncwarp();
-  const RxRange ir = rx_interior(p);
-  const u32 *gb = p.pf_gbits + (i64)G::GID * p.pf_ntiles;
-  const u32 *mm = p.pf_mmask + (i64)G::GID * 32 * p.pf_ntiles;
-  auto frame_blocks = [&](i64 w, i64 &b0, i64 &b1) {
-    i64 flo = (w * Bw - Lw) * 32, fhi = flo + 1024 * K;
-    if (flo < p.avail_lo) flo = p.avail_lo;
-    if (fhi > p.avail_hi) fhi = p.avail_hi;
-    if (fhi <= flo) fhi = flo + 1;
-    b0 = (flo - p.avail_lo) >> 10;
-    b1 = (fhi - 1 - p.avail_lo) >> 10;
-  };
-  i64 bmax = 0;
-  if (w_begin < w_end) {
-    i64 t0;
-    frame_blocks(w_end - 1, t0, bmax);
-  }
-  auto pending = [&](const u32 *a) -> bool {
-    if (NS == 0) return false;
-    bool any = false;
-    for (int s = (int)c.lane; s < NS; s += 32) any = any || a[s] != 0u;
-    return __any_sync(RX_FULL, any);
-  };
-  // first window >= w whose frame holds a factor of the group (w_end if none)
-  auto next_hit = [&](i64 w) -> i64 {
-    if (w >= w_end) return w_end;
-    if (G::ALWAYS != 0u) return w;
-    i64 b0, b1;
-    frame_blocks(w, b0, b1);
-    const i64 b = rx_pf_next(gb, b0, bmax, c.lane);
-    if (b > bmax) return w_end;
-    if (b <= b1) return w;
-    const i64 pos = p.avail_lo + b * RX_PF_BLK;
-    const i64 wn = rx_floor_div(rx_floor_div(pos, 32) + Lw - 32 * K, Bw) + 1;
-    const i64 r = wn > w + 1 ? wn : w + 1;
-    return r < w_end ? r : w_end;
-  };
-  i64 staged = -1;  // window whose bytes are in flight / in tbuf (-1: none)
-  u32 phase = 0;
-  auto stage = [&](i64 w) {
-    const i64 f = w * Bw - Lw;
-    if (w < w_end && f >= ir.lo && f + 32 * K <= ir.hi) {
-      __syncwarp();
-      if (c.lane == 0) rx_bulk_load(tbuf, p.in + f * 32, WB, bar);
-      staged = w;
-    }
-  };
-  auto retire = [&]() {  // wait for the copy in flight (keeps the mbarrier phase in step)
-    rx_mbar_wait(bar, phase);
-    phase ^= 1u;
-    staged = -1;
-  };
-  i64 w = pending(st) ? w_begin : next_hit(w_begin);
-  if (w < w_end) stage(w);
-  while (w < w_end) {
-    const bool pend_in = pending(st);
-    if (p.stats && c.lane == 0) atomicAdd(&p.stats[3], 1ull);
-    const i64 fword = w * Bw - Lw;
-    if (staged == w) {
-      retire();
-      const uint4 *q = reinterpret_cast<const uint4 *>(tbuf + c.lane * (32u * K));
-#pragma unroll
-      for (int k = 0; k < K; ++k) {
-        const uint4 a0 = q[2 * k], a1 = q[2 * k + 1];
-        xr[k][0] = a0.x; xr[k][1] = a0.y; xr[k][2] = a0.z; xr[k][3] = a0.w;
-        xr[k][4] = a1.x; xr[k][5] = a1.y; xr[k][6] = a1.z; xr[k][7] = a1.w;
-      }
-    } else {
-      if (staged >= 0 && staged < w) retire();  // a stale guess: drain it
-      rx_fetch<K>(p, ir, c.lane, xr, fword);
-    }
-    // guess the next window and start its copy before the body runs
-    if (staged < 0) {
-      const i64 guess = pend_in ? w + 1 : next_hit(w + 1);
-      stage(guess);
-    }
-    i64 b0, b1;
-    frame_blocks(w, b0, b1);
-    u32 mine = 0u;
-    for (i64 b = b0 + c.lane; b <= b1; b += 32)
-      if ((gb[b >> 5] >> (b & 31)) & 1u) mine |= mm[b];
-    const u32 rmask = __reduce_or_sync(RX_FULL, mine);
-    if (p.stats && c.lane == 0) {
-      atomicAdd(&p.stats[0], 1ull);
-      if (rmask == 0u) atomicAdd(&p.stats[1], 1ull);
-      atomicAdd(&p.stats[2], (u64)__popc(rmask));
-    }
-    c.cw = (u32)((len_words - w * Bw) < Bw ? (len_words - w * Bw) : Bw);
-    c.word0 = fword;
-    rx_unpack<K>(p, ir, c, xr, pl, fword);
-    rx_commit_mask(p, ir, c, Lw, fword);
-    if (NS > 0) rx_state_zero(nst, NS, c.lane);
-    G::body_i(c, pl, st, nst, rmask);
-    u32 *t = st;
-    st = nst;
-    nst = t;
-    __syncwarp();
-    w = pending(st) ? w + 1 : next_hit(w + 1);
-  }
-  if (staged >= 0) retire();
-  if (!live) return;
-  if (NS > 0) {
-    u32 *dst = p.seg_state + ((i64)seg * G::NG + G::GID) * G::NSMAX;
-    for (int s = (int)c.lane; s < NS; s += 32) dst[s] = st[s];
-    if (p.st_out && w_end == nwin)
-      for (int s = (int)c.lane; s < NS; s += 32) p.st_out[G::SBASE + s] = st[s];
-  }
-  rx_flush<G>(p, c);
-}
-
-// Cluster-major sparse pass 1 (the default).  The
-// segment is walked once per factor cluster of the group, running only that
-// cluster's out-of-line code (G::cbody) in the windows whose frame holds one
-// of its factors or into which its own state flows.  A cluster's code stays
-// in the SM's instruction caches across consecutive windows (one straight-
-// line body per window over the whole group thrashed them: the top stall was
-// "no instruction"), at the price of re-loading and re-transposing a window
-// for each cluster that runs in it.  Clusters own disjoint state slots, so
-// running them one after the other over the segment computes exactly what
-// the window-major order computes.  With cm_sync the CTA's warps (same group,
-// consecutive segments) step from cluster to cluster together.
-template <class G>
-DEV void rx_run_segment_cm(const RxParams &p, int seg, u64 *acc, u32 *sst, unsigned char *tbuf, u64 *bar,
-                           unsigned char *lb) {
-  constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw;
-  constexpr u32 WB = 1024u * K;
-  const i64 len_words = rx_div_up(p.len, 32);
-  const i64 nwin = rx_div_up(len_words, Bw);
-  const i64 w_begin = (i64)seg * p.sw;
-  const bool live = w_begin < nwin || seg == 0;
-  const i64 w_end = !live ? w_begin : (w_begin + p.sw < nwin ? w_begin + p.sw : nwin);
-  Ctx<K> c;
-  rx_ctx_init<G>(p, c, acc, lb);
-  u32 pl[8][K];
-  u32 xr[K][8];
-  u32 *st = sst, *nst = sst + G::NSMAX;
-  if (c.lane == 0) rx_mbar_init(bar, 1);
-  __syncwarp();
-  const RxRange ir = rx_interior(p);
-  const u32 *gb = p.pf_gbits + (i64)G::GID * p.pf_ntiles;
-  const u32 *mm = p.pf_mmask + (i64)G::GID * 32 * p.pf_ntiles;
-  auto frame_blocks = [&](i64 w, i64 &b0, i64 &b1) {
-    i64 flo = (w * Bw - Lw) * 32, fhi = flo + 1024 * K;
-    if (flo < p.avail_lo) flo = p.avail_lo;
-    if (fhi > p.avail_hi) fhi = p.avail_hi;
-    if (fhi <= flo) fhi = flo + 1;
-    b0 = (flo - p.avail_lo) >> 10;
-    b1 = (fhi - 1 - p.avail_lo) >> 10;
-  };
-  i64 bmax = 0;
-  if (w_begin < w_end) {
-    i64 t0;
-    frame_blocks(w_end - 1, t0, bmax);
-  }
-  // members of the group whose factor occurs in window w's frame
-  auto frame_hits = [&](i64 w) -> u32 {
-    i64 b0, b1;
-    frame_blocks(w, b0, b1);
-    u32 mine = 0u;
-    for (i64 b = b0 + c.lane; b <= b1; b += 32)
-      if ((gb[b >> 5] >> (b & 31)) & 1u) mine |= mm[b];
-    return __reduce_or_sync(RX_FULL, mine);
-  };
-  // first window >= w whose frame holds a factor of the group (w_end if none)
-  auto next_group_hit = [&](i64 w) -> i64 {
-    if (w >= w_end) return w_end;
-    i64 b0, b1;
-    frame_blocks(w, b0, b1);
-    const i64 b = rx_pf_next(gb, b0, bmax, c.lane);
-    if (b > bmax) return w_end;
-    if (b <= b1) return w;
-    const i64 pos = p.avail_lo + b * RX_PF_BLK;
-    const i64 wn = rx_floor_div(rx_floor_div(pos, 32) + Lw - 32 * K, Bw) + 1;
-    const i64 r = wn > w + 1 ? wn : w + 1;
-    return r < w_end ? r : w_end;
-  };
-  i64 staged = -1;
-  u32 phase = 0;
-  auto stage = [&](i64 w) {
-    const i64 f = w * Bw - Lw;
-    if (w < w_end && f >= ir.lo && f + 32 * K <= ir.hi) {
-      __syncwarp();
-      if (c.lane == 0) rx_bulk_load(tbuf, p.in + f * 32, WB, bar);
-      staged = w;
-    }
-  };
-  auto retire = [&]() {
-    rx_mbar_wait(bar, phase);
-    phase ^= 1u;
-    staged = -1;
-  };
-  for (int ci = 0; ci < G::NC; ++ci) {
-    const int s0 = G::cslot(ci), s1 = G::cslot(ci + 1);
-    const u32 cm = G::cmask(ci);
-    const bool always = G::calways(ci);
-    for (int s = s0 + (int)c.lane; s < s1; s += 32) st[s] = (seg == 0 && p.st_in) ? p.st_in[G::SBASE + s] : 0u;
-    __syncwarp();
-    auto pending = [&](const u32 *a) -> bool {
-      bool any = false;
-      for (int s = s0 + (int)c.lane; s < s1; s += 32) any = any || a[s] != 0u;
-      return __any_sync(RX_FULL, any);
-    };
-    // first window >= w in which this cluster must run (no state pending)
-    auto next_c = [&](i64 w) -> i64 {
-      if (always) return w < w_end ? w : w_end;
-      for (;;) {
-        w = next_group_hit(w);
-        if (w >= w_end) return w_end;
-        if (frame_hits(w) & cm) return w;
-        ++w;
-      }
-    };
-    i64 w = pending(st) ? w_begin : next_c(w_begin);
-    if (w < w_end) stage(w);
-    while (w < w_end) {
-      const bool pend_in = pending(st);
-      const i64 fword = w * Bw - Lw;
-      if (staged == w) {
-        retire();
-        const uint4 *q = reinterpret_cast<const uint4 *>(tbuf + c.lane * (32u * K));
-#pragma unroll
-        for (int k = 0; k < K; ++k) {
-          const uint4 a0 = q[2 * k], a1 = q[2 * k + 1];
-          xr[k][0] = a0.x; xr[k][1] = a0.y; xr[k][2] = a0.z; xr[k][3] = a0.w;
-          xr[k][4] = a1.x; xr[k][5] = a1.y; xr[k][6] = a1.z; xr[k][7] = a1.w;
-        }
-      } else {
-        if (staged >= 0 && staged < w) retire();
-        rx_fetch<K>(p, ir, c.lane, xr, fword);
-      }
-      if (staged < 0) stage(pend_in ? w + 1 : next_c(w + 1));
-      const u32 rmask = frame_hits(w) & cm;
-      if (p.stats && c.lane == 0) {
-        atomicAdd(&p.stats[0], 1ull);
-        if (rmask == 0u) atomicAdd(&p.stats[1], 1ull);
-        atomicAdd(&p.stats[2], (u64)__popc(rmask));
-        atomicAdd(&p.stats[3], 1ull);
-      }
-      c.cw = (u32)((len_words - w * Bw) < Bw ? (len_words - w * Bw) : Bw);
-      c.word0 = fword;
-      rx_unpack<K>(p, ir, c, xr, pl, fword);
-      rx_commit_mask(p, ir, c, Lw, fword);
-      for (int s = s0 + (int)c.lane; s < s1; s += 32) nst[s] = 0u;
-      __syncwarp();
-      G::cbody(ci, c, pl, st, nst, rmask);
-      u32 *t = st;
-      st = nst;
-      nst = t;
-      __syncwarp();
-      w = pending(st) ? w + 1 : next_c(w + 1);
-    }
-    if (staged >= 0) retire();
-    if (live && s1 > s0) {
-      u32 *dst = p.seg_state + ((i64)seg * G::NG + G::GID) * G::NSMAX;
-      for (int s = s0 + (int)c.lane; s < s1; s += 32) dst[s] = st[s];
-      if (p.st_out && w_end == nwin)
-        for (int s = s0 + (int)c.lane; s < s1; s += 32) p.st_out[G::SBASE + s] = st[s];
-    }
-    __syncwarp();
-    if (p.cm_sync) __syncthreads();
-  }
-  if (!live) return;
-  rx_flush<G>(p, c);
 }

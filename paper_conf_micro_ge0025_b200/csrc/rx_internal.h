@@ -5,6 +5,7 @@
 // program grammar P:L118 (Listing 2 lost).
 #pragma once
 #include <cstdint>
+#include <map>
 #include <memory>
 #include <string>
 #include <vector>
@@ -137,6 +138,7 @@ struct Cluster {
   RegexIR ir;                // shared IR of the members (lower_cluster)
   int slot_base = 0;         // first state slot of the cluster in the group
   bool always = false;       // members without a factor: runs in every window
+  bool bcap = false;         // every member has output factors: may run output-gated (mode B)
 };
 
 struct Group {
@@ -148,30 +150,52 @@ struct Group {
   int nslots = 0;
   std::vector<int> slot_base;  // per member regex
   double cost = 0;
+  int out_delta = 0;         // max output-factor distance of a member (bytes; the halo covers it)
 };
 
 // Cross-regex literal prefilter (rx_prefilter.cpp).
+// A factor is a window of up to 16 fixed-offset byte positions that every
+// (partial) match must contain: each position is an exact byte, a byte up to
+// one bit (e.g. [Ss]), or any byte.  Its *anchor* is a k-gram (2 <= k <= 4)
+// of consecutive narrow positions inside the window, found by hashing; the
+// whole window is then compared.
 struct FactorGram {
   uint32_t gram, mask;  // bytes of the k-gram in the top k bytes of a little-endian u32 window
   int k;
   bool operator==(const FactorGram &o) const { return gram == o.gram && mask == o.mask; }
 };
 struct Factor {
-  std::vector<FactorGram> grams;
-  double score = 0;  // estimated occurrences per position (ranking only)
+  std::vector<ByteSet> win;       // the window's positions (<= 16)
+  std::vector<FactorGram> grams;  // anchor alternatives (chosen by build_prefilter)
+  int ae = 0;                     // window index of the anchor's last byte
+  uint8_t xv[16] = {0}, xm[16] = {0};  // window bytes [e - ae, e - ae + 16): (byte & xm) == xv
+  double score = 0;               // estimated occurrences per position (ranking only)
 };
 struct Prefilter {
   int nfactor = 0;
-  std::vector<uint32_t> blob;  // device table layout: see RxParams::pf_tab (rx_device.cuh)
-  uint32_t o_ent = 0, o_fgoff = 0, o_fgent = 0;  // o_ent: the gram hash table
-  uint32_t hbits = 0;                            // log2 of its slots
+  std::vector<uint32_t> blob;  // device table layout: see rx_prefilter_run (rx_device.cuh)
+  uint32_t b4bits = 0;         // log2 bits of the 4-gram Bloom filter
+  uint32_t o_b3 = 0, o_b2 = 0; // word offsets of the 3-gram Bloom / bigram bitmap (0 = none)
+  uint32_t o_ht = 0, hbits = 0;  // anchor hash table {gram, k<<1|1, first ext, n ext}, log2 slots
+  uint32_t o_ext = 0;          // extension entries {ae, v[4], m[4], fid}
+  uint32_t o_fgoff = 0, o_fgent = 0;  // factor -> {group, member mask, kind} triples
+  uint32_t smem_words = 0;     // leading words staged in shared memory (Bloom filters + bitmap)
 };
-// Returns false if the regex has no usable factor (it then always runs).
-bool regex_factor(const Ast &a, Factor &f);
+// Per-regex factors.  first: prefix factors -- one of them lies inside every
+// partial match that produces output or reaches a state slot (empty: the
+// regex runs in every window).  out: output factors -- one of them ends at
+// most out_delta bytes before every match end (empty: none; the regex then
+// cannot run in output-gated mode B).
+struct RegexFactors {
+  std::vector<int> first, out;
+  int out_delta = 0;
+};
 
 struct CompiledSet {
-  std::vector<int> factor_of;     // per regex: factor id or -1 (always runs)
+  std::vector<int> factor_of;     // per regex: clustering key of its first-factor set, -1 = none (always runs)
+  std::vector<RegexFactors> rf;   // per regex
   std::vector<Factor> factors;
+  std::map<std::vector<std::vector<uint64_t>>, int> factor_ix;  // factor window -> id (deduplication)
   Prefilter pf;
   bool use_pf = false;
   std::vector<RegexIR> irs;
@@ -180,13 +204,19 @@ struct CompiledSet {
   std::string info;
 };
 
+// First and output factors of one regex, added to cs.factors (deduplicated).
+void regex_factors(const Ast &a, CompiledSet &cs, RegexFactors &rf);
+
 // CUDA C sources: one relocatable unit per group + the kernel unit; linked
 // into one module with nvJitLink.
 std::string emit_group_unit(CompiledSet &cs, int gi);
 std::string emit_kernel_unit(CompiledSet &cs);
 int lit_scratch_bytes(const CompiledSet &cs);  // per-warp shared bytes of the literal-run scratch
+int max_words_per_lane(const CompiledSet &cs);
+size_t warp_smem_bytes(const CompiledSet &cs);  // per-warp shared bytes of pass 1 / fix-up
 bool plan_groups(CompiledSet &cs, int group_size, int force_K, std::string &why);
 void build_prefilter(CompiledSet &cs);
+std::string factor_info(const CompiledSet &cs, int r);  // "first [...] out [...]" (rx_program_info)
 // Partition each group's members into clusters (same factor, or no factor)
 // and lower each cluster jointly; recomputes the group's state slots.
 bool build_clusters(CompiledSet &cs, const std::vector<const Ast *> &asts, const LowerOptions &opt,

@@ -606,11 +606,9 @@ bool plan_groups(CompiledSet &cs, int group_size, int force_K, std::string &why)
   for (auto &r : cs.irs) total_instr += r.n_instr;
   if (group_size <= 0 || group_size > 32) group_size = 32;  // member masks are 32-bit
   // bounds one NVRTC unit (compile time) and the group's code size (the
-  // SM's instruction caches hold one group's program); RX_GROUP_INSTR
-  // overrides (experiments)
-  size_t max_instr = 1500;
-  if (const char *e = getenv("RX_GROUP_INSTR"))
-    if (atoi(e) > 0) max_instr = (size_t)atoi(e);
+  // SM's instruction caches hold one group's program; measured flat over
+  // 600-3000)
+  const size_t max_instr = 1500;
   cs.groups.clear();
   Group g;
   size_t gi = 0;
@@ -632,10 +630,17 @@ bool plan_groups(CompiledSet &cs, int group_size, int force_K, std::string &why)
     gr.nslots = 0;
     gr.slot_base.clear();
     gr.always = 0;
+    gr.out_delta = 0;
     for (int r : gr.regexes) {
       const RegexIR &ir = cs.irs[r];
       if (fac(r) < 0) gr.always |= 1u << gr.slot_base.size();
       L = std::max(L, (ir.lb + 31) / 32);
+      // mode B (output-gated) needs every output-factor anchor of a match
+      // ending in the committed range inside the frame: Lw words >= delta
+      if (!cs.rf.empty() && !cs.rf[r].out.empty()) {
+        gr.out_delta = std::max(gr.out_delta, cs.rf[r].out_delta);
+        L = std::max(L, (cs.rf[r].out_delta + 31) / 32);
+      }
       R = std::max(R, (std::max(ir.rb, ir.rb_state) + 31) / 32);
       gr.slot_base.push_back(gr.nslots);
       gr.nslots += ir.nslots;
@@ -669,17 +674,21 @@ bool build_clusters(CompiledSet &cs, const std::vector<const Ast *> &asts, const
                     std::string &why) {
   for (auto &g : cs.groups) {
     g.clusters.clear();
-    std::map<int, int> by_factor;  // factor id (-1 = none) -> cluster
+    // cluster key: (first-factor set, has output factors) -- a cluster runs
+    // output-gated (mode B) only if all of its members can
+    std::map<std::pair<int, bool>, int> by_factor;
     for (size_t m = 0; m < g.regexes.size(); ++m) {
       const int r = g.regexes[m];
       const int f = cs.factor_of.empty() ? -1 : cs.factor_of[r];
-      auto it = by_factor.find(f);
+      const bool bc = !cs.rf.empty() && !cs.rf[r].out.empty();
+      auto it = by_factor.find({f, bc});
       int ci;
       if (it == by_factor.end()) {
         ci = (int)g.clusters.size();
-        by_factor[f] = ci;
+        by_factor[{f, bc}] = ci;
         g.clusters.emplace_back();
         g.clusters.back().always = f < 0;
+        g.clusters.back().bcap = bc;
       } else {
         ci = it->second;
       }

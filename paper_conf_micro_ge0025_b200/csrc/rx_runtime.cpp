@@ -206,10 +206,14 @@ bool nvrtc_compile(const std::string &src, int max_regs, bool use_cache, std::st
 // ---------------------------------------------------------------------------
 // program
 // ---------------------------------------------------------------------------
+constexpr int kPass1Warps = 16;  // one CTA = one SM's worth of warps, one group (lockstep)
+constexpr int kFixupWarps = 4;
+constexpr int kPrefilterWarps = 8;
+constexpr size_t kMaxSmem = 232448;  // opt-in dynamic shared memory per block (227 KB)
 struct RxModule {
   int g_begin = 0, g_end = 0;  // group range
   int ns_max = 1, nr_max = 1;
-  int lit_bytes = 0;  // per-warp literal-run scratch (rx_codegen.cpp lit_scratch_bytes)
+  size_t warp_smem = 0;  // per-warp shared bytes of pass 1 / fix-up (rx_codegen.cpp warp_smem_bytes)
   bool any_state = false;
   std::string source;
   std::vector<std::string> units;  // relocatable sm_100a cubins (groups + kernels)
@@ -223,6 +227,7 @@ struct RxModule {
 
 struct rx_program {
   rx::CompiledSet cs;
+  uint32_t flags = 0;  // rx_options.flags
   std::vector<RxModule> mods;
   uint32_t n_regex = 0;
   uint32_t state_words = 0;
@@ -248,7 +253,7 @@ struct rx_program {
 
 namespace {
 // scratch slots of one rx_match call
-enum { SC_STATUS = 0, SC_SEGSTATE = 1, SC_PF = 2, SC_TASK = 3, SC_FIX = 4 };
+enum { SC_STATUS = 0, SC_SEGSTATE = 1, SC_PF = 2, SC_FIX = 3 };
 void *scratch_get(rx_program *p, cudaStream_t s, int slot, size_t bytes) {
   std::lock_guard<std::mutex> lk(p->mu);
   auto &e = p->scratch[{(void *)s, slot}];
@@ -280,6 +285,18 @@ uint32_t rx_kernels_per_match(const rx_program *p) {
   return n;
 }
 const char *rx_program_info(const rx_program *p) { return p ? p->info.c_str() : ""; }
+
+size_t rx_prefilter_table(const rx_program *p, const uint32_t **blob, uint32_t *hdr) {
+  if (!p || !p->cs.use_pf) return 0;
+  const rx::Prefilter &pf = p->cs.pf;
+  if (blob) *blob = pf.blob.data();
+  if (hdr) {
+    const uint32_t h[12] = {pf.smem_words, pf.b4bits, pf.hbits >> 8, pf.hbits & 255u, pf.o_b3, pf.o_b2,
+                            pf.o_ht,       pf.o_ext,  pf.o_fgoff,   pf.o_fgent,       (uint32_t)pf.nfactor, 0u};
+    memcpy(hdr, h, sizeof h);
+  }
+  return pf.blob.size();
+}
 
 rx_status rx_set_profiling(rx_program *p, int on) {
   if (!p) return fail(RX_EINVAL, "null program");
@@ -342,13 +359,25 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
   lo.rebalance = (o.flags & RX_F_REBALANCE) && !(o.flags & RX_F_NO_REBALANCE);
   int max_regs = o.max_regs ? (int)o.max_regs : 128;
 
+  if (o.words_per_lane != 0 && o.words_per_lane != 1 && o.words_per_lane != 2 && o.words_per_lane != 4 &&
+      o.words_per_lane != 8) {
+    if (err) {
+      err->pattern_index = 0;
+      err->byte_offset = 0;
+      snprintf(err->msg, sizeof err->msg, "words_per_lane must be 0, 1, 2, 4 or 8");
+    }
+    return fail(RX_EINVAL, "words_per_lane must be 0, 1, 2, 4 or 8");
+  }
+
   auto *p = new rx_program();
   p->n_regex = n_patterns;
+  p->flags = o.flags;
   p->cs.irs.resize(n_patterns);
   p->cs.factor_of.assign(n_patterns, -1);
+  p->cs.rf.assign(n_patterns, rx::RegexFactors());
   std::vector<rx::AstP> asts(n_patterns);
   const bool use_pf = !(o.flags & RX_F_NO_PREFILTER);
-  std::map<std::vector<uint32_t>, int> factor_ix;
+  std::map<std::vector<int>, int> first_key;  // first-factor set -> clustering key
   for (uint32_t i = 0; i < n_patterns; ++i) {
     std::string pat(patterns[i], pattern_lens[i]);
     rx::ParseError pe;
@@ -371,22 +400,16 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
       delete p;
       return fail(RX_ETOOBIG, "pattern " + std::to_string(i) + ": expansion too large");
     }
-    {
-      rx::Factor f;
-      int fid = -1;
-      if (use_pf && rx::regex_factor(*ast, f)) {
-        std::vector<uint32_t> key;
-        for (auto &g : f.grams) key.insert(key.end(), {g.gram, g.mask});
-        auto it = factor_ix.find(key);
-        if (it == factor_ix.end()) {
-          fid = (int)p->cs.factors.size();
-          factor_ix[key] = fid;
-          p->cs.factors.push_back(f);
-        } else {
-          fid = it->second;
-        }
+    if (use_pf) {
+      rx::regex_factors(*ast, p->cs, p->cs.rf[i]);
+      if (o.flags & RX_F_NO_MODEB) p->cs.rf[i].out.clear();
+      const auto &fs = p->cs.rf[i].first;
+      if (!fs.empty()) {
+        auto it = first_key.find(fs);
+        const int key = it == first_key.end() ? (int)first_key.size() : it->second;
+        if (it == first_key.end()) first_key[fs] = key;
+        p->cs.factor_of[i] = key;
       }
-      p->cs.factor_of[i] = fid;
     }
     {
       rx::LowerOptions ro = lo;
@@ -411,7 +434,9 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
     delete p;
     return fail(RX_ETOOBIG, why);
   }
-  p->cs.use_pf = !p->cs.factors.empty();
+  p->cs.use_pf = use_pf && !p->cs.factors.empty();
+  if (!p->cs.use_pf)  // no factor at all: every group runs dense, nothing is output-gated
+    for (auto &rf : p->cs.rf) rf = rx::RegexFactors();
   {
     std::vector<const rx::Ast *> ap;
     for (auto &a : asts) ap.push_back(a.get());
@@ -435,7 +460,9 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
   for (int gi = 0; gi < G; ++gi) {
     auto &g = p->cs.groups[gi];
     info << "group " << gi << ": regexes=" << g.regexes.size() << " K=" << g.K << " Lw=" << g.Lw << " Rw=" << g.Rw
-         << " Bw=" << g.Bw << " slots=" << g.nslots << "\n";
+         << " Bw=" << g.Bw << " slots=" << g.nslots << " clusters=" << g.clusters.size() << " members=";
+    for (size_t m = 0; m < g.regexes.size(); ++m) info << (m ? "," : "") << g.regexes[m];
+    info << "\n";
     p->lookback = std::max<uint32_t>(p->lookback, 32u * (uint32_t)g.Lw);
     p->lookahead = std::max<uint32_t>(p->lookahead, 32u * (uint32_t)g.Rw);
     mm.ns_max = std::max(mm.ns_max, g.nslots);
@@ -444,22 +471,30 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
     sbase += (uint32_t)g.nslots;
   }
   p->state_words = sbase;
-  mm.lit_bytes = rx::lit_scratch_bytes(p->cs);
   info << "prefilter: " << (p->cs.use_pf ? "on" : "off") << ", factors=" << p->cs.factors.size() << "\n";
   for (uint32_t i = 0; i < n_patterns; ++i) {
-    const int f = p->cs.factor_of[i];
     info << "regex " << i << ": factor ";
-    if (f < 0) info << "none (always runs)";
-    else {
-      info << f << " (" << p->cs.factors[f].grams.size() << " grams, k=" << p->cs.factors[f].grams[0].k
-           << ", score=" << p->cs.factors[f].score << ") grams=";
-      char hx[24];
-      for (auto &g : p->cs.factors[f].grams) {
-        snprintf(hx, sizeof hx, "%08x/%d,", g.gram, g.k);
-        info << hx;
-      }
-    }
+    if (p->cs.use_pf) info << rx::factor_info(p->cs, (int)i);
+    else info << "none (always runs)";
     info << "\n" << rx::dump_ir(p->cs.irs[i]);
+  }
+  // shared memory: pass 1 / fix-up per warp, prefilter per CTA (ADVICE r1:
+  // a program whose layout exceeds the opt-in limit must fail here, not at
+  // every launch)
+  mm.warp_smem = rx::warp_smem_bytes(p->cs);
+  if (mm.warp_smem * kPass1Warps > kMaxSmem) {
+    delete p;
+    return fail(RX_ETOOBIG, "pass-1 shared memory " + std::to_string(mm.warp_smem * kPass1Warps) +
+                                " B exceeds the 227 KB per-block limit (fewer state slots / regexes per group, or "
+                                "smaller words_per_lane)");
+  }
+  if (p->cs.use_pf) {
+    const size_t pfb =
+        4 * (((size_t)p->cs.pf.smem_words + 3) & ~(size_t)3) + 4 * 64 * (size_t)G + 4 * 96 * kPrefilterWarps;
+    if (pfb > kMaxSmem) {
+      delete p;
+      return fail(RX_ETOOBIG, "prefilter shared memory " + std::to_string(pfb) + " B exceeds the 227 KB limit");
+    }
   }
   p->info = info.str();
   std::vector<std::string> srcs(G + 1), cubins(G + 1), logs(G + 1);
@@ -508,7 +543,7 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
 // ---------------------------------------------------------------------------
 namespace {
 
-struct RxParamsHost {  // must mirror RxParams in rx_device.cuh
+struct RxParamsHost {  // must mirror RxParams in rx_device.cuh (tests/test_library_cpu.py checks the fields)
   const unsigned char *in;
   long long avail_lo, avail_hi;
   long long valid_lo, valid_hi;
@@ -528,28 +563,24 @@ struct RxParamsHost {  // must mirror RxParams in rx_device.cuh
   int aligned;
   int mode;
   int accumulate;
-  int lockstep;
+  int modeb;
   const unsigned int *pf_tab;
-  unsigned int pf_words;
-  unsigned int pf_o_ent, pf_o_fgoff, pf_o_fgent;
-  unsigned int pf_hbits;
-  int pf_tab_smem;
+  unsigned int pf_words, pf_smem_words;
+  unsigned int pf_b4bits, pf_b3bits, pf_hbits;
+  unsigned int pf_o_b3, pf_o_b2, pf_o_ht, pf_o_ext, pf_o_fgoff, pf_o_fgent;
   unsigned int *pf_gbits;
   unsigned int *pf_mmask;
+  unsigned int *pf_omask;
+  unsigned int *pf_cnt;
   long long pf_ntiles;
   int pf_on;
-  int pf_aligned;
   unsigned long long *stats;
-  int dbg;
   unsigned long long *matches;
   unsigned long long match_cap;
   unsigned long long *match_total;
   int fix_phase;
   unsigned int *seg_fix;
   unsigned int *seg_nc;
-  unsigned long long *task_ctr;
-  int cmajor;
-  int cm_sync;
 };
 
 rx_status ensure_loaded(rx_program *p, int &device) {
@@ -597,35 +628,38 @@ rx_status ensure_loaded(rx_program *p, int &device) {
   return RX_OK;
 }
 
-constexpr int kPass1Warps = 16;  // one CTA = one SM's worth of warps, one group (lockstep)
-constexpr int kFixupWarps = 4;
-
 rx_status launch(rx_program *p, RxModule &m, CUfunction f, long long blocks, int warps_per_block,
                  const RxParamsHost &prm, cudaStream_t s) {
   Drv &d = drv();
   if (blocks <= 0) return RX_OK;
+  if (blocks > 0x7fffffffLL) return fail(RX_EINVAL, "grid too large");
+  // shared memory: pass 1 / fix-up = per-warp layout of rx_codegen.cpp
+  // emit_group_unit; prefilter = [filters | 2 x NG x 32 member masks | hit queues]
+  size_t bytes = (size_t)warps_per_block * m.warp_smem;
+  if (f == m.prefilter)
+    bytes = 4 * (((size_t)prm.pf_smem_words + 3) & ~(size_t)3) + 4 * 64 * (size_t)(m.g_end - m.g_begin) +
+            4 * 96 * (size_t)warps_per_block;
+  if (bytes > kMaxSmem) return fail(RX_ETOOBIG, "shared memory layout exceeds 227 KB");
+  const unsigned smem = (unsigned)bytes;
+  if (smem > 48 * 1024 &&
+      d.FuncSetAttribute(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)smem) != CUDA_SUCCESS)
+    return fail(RX_ECUDA, "cuFuncSetAttribute(max dynamic shared memory = " + std::to_string(smem) + ") failed");
+  bool prof;
+  {
+    std::lock_guard<std::mutex> lk(p->mu);
+    prof = p->prof;
+  }
   rx_program::Ev ev{f == m.prefilter ? 0 : (f == m.pass1 ? 1 : 2), nullptr, nullptr};
-  if (p->prof) {
+  if (prof) {
     cudaEventCreate(&ev.a);
     cudaEventCreate(&ev.b);
     cudaEventRecord(ev.a, s);
   }
-  if (blocks > 0x7fffffffLL) return fail(RX_EINVAL, "grid too large");
-  // must match the layout emitted in rx_codegen.cpp (accumulators | state |
-  // TMA window staging | mbarriers); the fix-up kernel uses the first two
-  const size_t wpb = (size_t)warps_per_block;
-  size_t bytes = wpb * 3 * m.nr_max * 8 + (((wpb * 4 * m.ns_max) + 3) & ~(size_t)3) * 4 + wpb * (size_t)m.lit_bytes;
-  if (f == m.pass1) bytes += wpb * 4096 + wpb * 16;
-  if (f == m.prefilter)
-    bytes = 4 * ((prm.pf_tab_smem ? ((prm.pf_words + 3) & ~3u) : 4096u) + 32 * (size_t)(m.g_end - m.g_begin) +
-                 96 * (size_t)warps_per_block);
-  unsigned smem = (unsigned)bytes;
-  if (smem > 48 * 1024) d.FuncSetAttribute(f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)smem);
   RxParamsHost local = prm;
   void *args[] = {&local};
   CUresult r =
       d.LaunchKernel(f, (unsigned)blocks, 1, 1, 32 * warps_per_block, 1, 1, smem, (CUstream)s, args, nullptr);
-  if (p->prof) {
+  if (prof) {
     cudaEventRecord(ev.b, s);
     std::lock_guard<std::mutex> lk(p->mu);
     p->prof_ev.push_back(ev);
@@ -644,6 +678,7 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
   if (out->d_bitstreams && out->pitch_words < (len + 31) / 32) return fail(RX_EINVAL, "pitch_words too small");
   if ((halo_left != 0 && halo_left < p->lookback) || (halo_right != 0 && halo_right < p->lookahead))
     return fail(RX_EINVAL, "halo smaller than rx_max_lookback / rx_max_lookahead");
+  if (out->d_matches && !out->d_match_total) return fail(RX_EINVAL, "d_matches needs d_match_total");
   int device = -1;
   rx_status s = ensure_loaded(p, device);
   if (s != RX_OK) return s;
@@ -680,24 +715,20 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
   prm.st_assumed = (const unsigned int *)st_assumed;
   prm.aligned = (((uintptr_t)d_input) & 15) == 0 ? 1 : 0;
   prm.accumulate = accumulate;
-  if (out->d_matches && !out->d_match_total) return fail(RX_EINVAL, "d_matches needs d_match_total");
   prm.matches = (unsigned long long *)out->d_matches;
   prm.match_cap = out->d_matches ? out->match_cap : 0;
   prm.match_total = (unsigned long long *)out->d_match_total;
-  {
-    const char *e = getenv("RX_LOCKSTEP");  // experiment knob: 0 = no per-window CTA barrier
-    prm.lockstep = (e && *e == '0') ? 0 : 1;
-  }
-  static unsigned int dummy_status_host = 0;
-  (void)dummy_status_host;
-  unsigned int *status_scratch = nullptr;
+  // mode B (output-gated clusters) only for a whole
+  // stream: its walk-back may read any earlier byte and reconstructs state
+  // from the stream start, so chunks (incoming / outgoing state) use mode A
+  prm.modeb = (mode == 0 && !st_in && !st_out && halo_left == 0) ? 1 : 0;
   if (!prm.status) {
-    if (!(status_scratch = (unsigned int *)scratch_get(p, stream, SC_STATUS, 256))) return fail(RX_ENOMEM, "status");
+    unsigned int *status_scratch = (unsigned int *)scratch_get(p, stream, SC_STATUS, 256);
+    if (!status_scratch) return fail(RX_ENOMEM, "status");
     cudaMemsetAsync(status_scratch, 0, 4, stream);
     prm.status = status_scratch;
   }
   const long long len_words = div_up((long long)len, 32);
-  const int G = (int)p->cs.groups.size();
   if (mode == 2) {
     prm.mode = 2;
     prm.sw = 1 << 30;
@@ -710,25 +741,13 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
     }
     return RX_OK;
   }
-  // segments: enough warps to fill the GPU several times over
+  // pass-1 geometry: CTAs of 16 warps, one group per CTA, 16 consecutive
+  // segments; ~16 waves of 148 CTAs so that the hardware CTA scheduler
+  // evens out the data-dependent work
+  const int G = (int)p->cs.groups.size();
   long long max_nwin = 0;
   for (auto &g : p->cs.groups) max_nwin = std::max(max_nwin, div_up(len_words, g.Bw));
-  // pass-1 CTAs: 16 segments of one group each; aim for ~4 waves of 148 SMs.
-  // Dynamic (sparse) mode: ~16 (group, segment) tasks per resident warp so
-  // that the dynamic queue evens out the data-dependent work
-  // experiment knobs: RX_DYNAMIC=1 persistent
-  // warps pulling (group, segment) tasks; RX_CMAJOR=0 window-major sparse
-  // pass; RX_CM_SYNC=0 no CTA barrier between clusters
-  const char *pls = getenv("RX_PF_LOCKSTEP"), *dys = getenv("RX_DYNAMIC");
-  const bool dynamic = p->cs.use_pf && !(pls && *pls == '1') && (dys && *dys == '1');
-  {
-    const char *e1 = getenv("RX_CMAJOR"), *e2 = getenv("RX_CM_SYNC");
-    prm.cmajor = (e1 && *e1 == '0') ? 0 : 1;
-    prm.cm_sync = (e2 && *e2 == '0') || dynamic ? 0 : 1;
-  }
-  long long waves = 16;  // RX_WAVES: pass-1 CTA waves per SM (measured best for the Snort-like set; knob)
-  if (const char *e = getenv("RX_WAVES"))
-    if (atoi(e) > 0) waves = atoi(e);
+  const long long waves = 16;
   const long long target_ctas = 148LL * waves;
   const long long cpg0 = std::max<long long>(1, div_up(target_ctas, std::max(G, 1)));
   long long sw = std::max<long long>(4, div_up(max_nwin, cpg0 * kPass1Warps));
@@ -737,6 +756,7 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
   prm.sw = (int)std::min<long long>(sw, 1 << 30);
   prm.nseg_max = (int)nseg_max;
   prm.mode = 0;
+  const bool stats_on = (p->flags & RX_F_STATS) != 0;
   for (auto &m : p->mods) {
     int mg = m.g_end - m.g_begin;
     unsigned int *seg_state = nullptr;
@@ -746,93 +766,78 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
     }
     prm.seg_state = seg_state;
     prm.mode = 0;
-    void *pf_scratch = nullptr;
+    prm.pf_on = 0;
     if (p->cs.use_pf) {
       const long long span = prm.avail_hi - prm.avail_lo;
       const long long ntiles = std::max<long long>(1, div_up(span, 32768));
-      const size_t gb_bytes = (size_t)4 * (size_t)ntiles * (size_t)mg;
-      const size_t bl_bytes = (size_t)4 * 32 * (size_t)ntiles * (size_t)mg;
-      if (!(pf_scratch = scratch_get(p, stream, SC_PF, gb_bytes + bl_bytes + 256)))
-        return fail(RX_ENOMEM, "prefilter scratch");
+      const size_t gb_bytes = ((size_t)4 * (size_t)ntiles * (size_t)mg + 255) & ~(size_t)255;
+      const size_t bl_bytes = ((size_t)4 * 32 * (size_t)ntiles * (size_t)mg + 255) & ~(size_t)255;
+      const size_t cnt_bytes = (size_t)4 * 64 * (size_t)mg;
+      char *pf_scratch = (char *)scratch_get(p, stream, SC_PF, gb_bytes + 2 * bl_bytes + cnt_bytes + 256);
+      if (!pf_scratch) return fail(RX_ENOMEM, "prefilter scratch");
+      const rx::Prefilter &pf = p->cs.pf;
       prm.pf_tab = (const unsigned int *)m.pf_mem;
-      prm.pf_words = (unsigned int)p->cs.pf.blob.size();
-      prm.pf_o_ent = p->cs.pf.o_ent;
-      prm.pf_o_fgoff = p->cs.pf.o_fgoff;
-      prm.pf_o_fgent = p->cs.pf.o_fgent;
-      prm.pf_hbits = p->cs.pf.hbits;
-      // shared memory: [table (or its 16 KiB bigram bitmap + rank) | NG x 32 member masks | hit queues]
-      const size_t fixed = 128ull * (size_t)mg + 6144;
-      prm.pf_tab_smem = 4ull * prm.pf_words + fixed <= 220 * 1024 ? 1 : 0;
-      if (!prm.pf_tab_smem && 16384 + fixed > 227 * 1024)
-        return fail(RX_ETOOBIG, "too many groups for the prefilter's shared member masks");
+      prm.pf_words = (unsigned int)pf.blob.size();
+      prm.pf_smem_words = pf.smem_words;
+      prm.pf_b4bits = pf.b4bits;
+      prm.pf_b3bits = pf.hbits >> 8;
+      prm.pf_hbits = pf.hbits & 255u;
+      prm.pf_o_b3 = pf.o_b3;
+      prm.pf_o_b2 = pf.o_b2;
+      prm.pf_o_ht = pf.o_ht;
+      prm.pf_o_ext = pf.o_ext;
+      prm.pf_o_fgoff = pf.o_fgoff;
+      prm.pf_o_fgent = pf.o_fgent;
       prm.pf_gbits = (unsigned int *)pf_scratch;
-      prm.pf_mmask = (unsigned int *)((char *)pf_scratch + ((gb_bytes + 255) & ~(size_t)255));
+      prm.pf_mmask = (unsigned int *)(pf_scratch + gb_bytes);
+      prm.pf_omask = (unsigned int *)(pf_scratch + gb_bytes + bl_bytes);
+      prm.pf_cnt = (unsigned int *)(pf_scratch + gb_bytes + 2 * bl_bytes);
       prm.pf_ntiles = ntiles;
       prm.pf_on = 1;
-      prm.pf_aligned = (((uintptr_t)(d_input - halo_left)) & 15) == 0 ? 1 : 0;
-      {
-        const char *e = getenv("RX_PF_LOCKSTEP");  // experiment knob
-        prm.lockstep = (e && *e == '1') ? 1 : 0;
-      }
-      s = launch(p, m, m.prefilter, std::min<long long>(ntiles, 148LL * 4), 16, prm, stream);
+      if (cudaMemsetAsync(prm.pf_cnt, 0, cnt_bytes, stream) != cudaSuccess) return fail(RX_ECUDA, "memset");
+      // 8-warp CTAs, several per SM (the verification of filter hits is a
+      // chain of dependent loads: more resident warps hide it)
+      s = launch(p, m, m.prefilter, std::min<long long>(ntiles, 148LL * 8), kPrefilterWarps, prm, stream);
       if (s != RX_OK) return s;
     }
     unsigned long long *stats = nullptr;
-    const char *se = getenv("RX_STATS");
-    if (se && *se == '1' && cudaMalloc((void **)&stats, 64) == cudaSuccess) cudaMemsetAsync(stats, 0, 64, stream);
+    const size_t stats_bytes = 8 * (8 + 4 * (size_t)mg);
+    if (stats_on && cudaMalloc((void **)&stats, stats_bytes) == cudaSuccess)
+      cudaMemsetAsync(stats, 0, stats_bytes, stream);
     prm.stats = stats;
-    {
-      const char *de = getenv("RX_DBG");  // timing experiments only: results are wrong when set
-      prm.dbg = (de && *de) ? atoi(de) : 0;
-    }
-    // sparse (prefilter, no lockstep): a persistent grid pulling (group,
-    // segment) tasks dynamically; otherwise the static group-per-CTA map
-    long long p1_blocks = cpg * mg;
-    void *tctr = nullptr;
-    {
-      if (dynamic && prm.pf_on && !prm.lockstep) {
-        if (!(tctr = scratch_get(p, stream, SC_TASK, 256))) return fail(RX_ENOMEM, "task counter");
-        cudaMemsetAsync(tctr, 0, 8, stream);
-        prm.task_ctr = (unsigned long long *)tctr;
-        p1_blocks = std::min<long long>(p1_blocks, 148LL);
-      }
-    }
-    s = launch(p, m, m.pass1, p1_blocks, kPass1Warps, prm, stream);
-    prm.task_ctr = nullptr;
+    s = launch(p, m, m.pass1, cpg * mg, kPass1Warps, prm, stream);
     prm.stats = nullptr;
     if (stats) {
-      unsigned long long h[8];
-      cudaMemcpyAsync(h, stats, 64, cudaMemcpyDeviceToHost, stream);
+      std::vector<unsigned long long> h(stats_bytes / 8);
+      cudaMemcpyAsync(h.data(), stats, stats_bytes, cudaMemcpyDeviceToHost, stream);
       cudaStreamSynchronize(stream);
-      fprintf(stderr, "[rx stats] groups=%d window_checks=%llu active=%llu state_only=%llu member_hits=%llu\n", mg,
-              h[3], h[0], h[1], h[2]);
+      fprintf(stderr, "[rx stats] groups=%d window_visits=%llu active=%llu member_hits=%llu walkbacks=%llu "
+              "walk_rounds=%llu\n", mg, h[3], h[0], h[2], h[4], h[5]);
+      for (int g = 0; g < mg; ++g)
+        fprintf(stderr, "[rx stats] group %d: active=%llu member_hits=%llu modeB_members=%llu\n", g, h[8 + 4 * g],
+                h[9 + 4 * g], h[10 + 4 * g]);
       cudaFree(stats);
     }
-    prm.pf_on = 0;
     if (s != RX_OK) return s;
     if (m.any_state) {
+      // carry fix-up, phase 1: one warp per (group, segment) in parallel;
+      // phase 2: one warp per group, only where a segment's carry outlived it.
+      // (pf_on stays set: the fix-up recomputes the mode-B choice from the
+      // prefilter's counts and leaves those clusters alone)
       prm.mode = 1;
-      const char *fe = getenv("RX_FIX_SERIAL");  // experiment knob: the one-warp-per-group serial fix-up
-      if (fe && *fe == '1') {
-        prm.fix_phase = 0;
+      void *fx = nullptr;
+      const size_t nc_bytes = 4ull * (size_t)nseg_max * (size_t)mg;
+      if (!(fx = scratch_get(p, stream, SC_FIX, bytes + nc_bytes + 256))) return fail(RX_ENOMEM, "fix-up scratch");
+      prm.seg_fix = (unsigned int *)fx;
+      prm.seg_nc = (unsigned int *)((char *)fx + ((bytes + 255) & ~(size_t)255));
+      cudaMemsetAsync(prm.seg_nc, 0, nc_bytes, stream);
+      prm.fix_phase = 1;
+      s = launch(p, m, m.fixup, div_up((long long)mg * nseg_max, kFixupWarps), kFixupWarps, prm, stream);
+      if (s == RX_OK) {
+        prm.fix_phase = 2;
         s = launch(p, m, m.fixup, div_up(mg, kFixupWarps), kFixupWarps, prm, stream);
-      } else {
-        // phase 1: one warp per (group, segment) in parallel; phase 2: one
-        // warp per group, only where a segment's carry outlived it
-        void *fx = nullptr;
-        const size_t nc_bytes = 4ull * (size_t)nseg_max * (size_t)mg;
-        if (!(fx = scratch_get(p, stream, SC_FIX, bytes + nc_bytes + 256))) return fail(RX_ENOMEM, "fix-up scratch");
-        prm.seg_fix = (unsigned int *)fx;
-        prm.seg_nc = (unsigned int *)((char *)fx + ((bytes + 255) & ~(size_t)255));
-        cudaMemsetAsync(prm.seg_nc, 0, nc_bytes, stream);
-        prm.fix_phase = 1;
-        s = launch(p, m, m.fixup, div_up((long long)mg * nseg_max, kFixupWarps), kFixupWarps, prm, stream);
-        if (s == RX_OK) {
-          prm.fix_phase = 2;
-          s = launch(p, m, m.fixup, div_up(mg, kFixupWarps), kFixupWarps, prm, stream);
-        }
-        prm.fix_phase = 0;
       }
+      prm.fix_phase = 0;
       if (s != RX_OK) return s;
     }
   }

@@ -9,6 +9,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 os.environ.setdefault("RX_CACHE_DIR", os.path.join(ROOT, ".rxcache"))
 
+import bench  # noqa: E402
 import gen  # noqa: E402
 import paper_conf_micro_ge0025_b200 as rx  # noqa: E402
 
@@ -22,5 +23,7 @@ SETS = {
 
 for name in sys.argv[1:] or list(SETS):
     t = time.time()
-    prog = rx.Program(SETS[name]())
+    prog = rx.Program(SETS[name](), **bench.PROGRAM_OPTS.get(name, {}))  # the bench's launch configuration
+    if name == "snort":
+        rx.Program(SETS[name]())  # the default geometry too (tests)
     print(f"{name}: {prog.n_regex} regexes, {prog.n_groups} groups, {time.time() - t:.1f} s", flush=True)

@@ -105,6 +105,58 @@ def _check(config, cap, prefix, windows, seed):
     assert int(counts.sum()) > 0
 
 
+def _golden(name):
+    """tests/golden/full_<name>.tsv (scripts/make_goldens.py: the CPU oracle
+    over the whole workload) -> (header dict, counts, d1, d2)"""
+    hdr, rows = {}, []
+    with open(os.path.join(ROOT, "tests", "golden", f"full_{name}.tsv")) as f:
+        for line in f:
+            if line.startswith("#"):
+                continue
+            parts = line.rstrip("\n").split("\t")
+            if len(parts) == 2:
+                hdr[parts[0]] = parts[1]
+            else:
+                rows.append([int(x) for x in parts])
+    a = np.array(rows, dtype=np.uint64)
+    return hdr, a[:, 1], a[:, 2], a[:, 3]
+
+
+def _sha(pats, data):
+    import hashlib
+    h = hashlib.sha256()
+    for p in pats:
+        h.update(len(p).to_bytes(8, "little"))
+        h.update(p)
+    return h.hexdigest(), hashlib.sha256(np.ascontiguousarray(data).data).hexdigest()
+
+
+@pytest.mark.parametrize("config", ["snort", "dotstar", "clamav"])
+def test_full_size_every_regex_vs_golden(config):
+    """Every regex of the config, over the WHOLE input, in the launch
+    configuration bench.py times: per-regex counts and both position digests
+    equal the CPU oracle's (tests/golden/full_<config>.tsv, written by
+    scripts/make_goldens.py, which calls only oracle/)."""
+    hdr, g_counts, g_d1, g_d2 = _golden(config)
+    pats, data, nbytes, _ = bench.load_workload(config)
+    ps, ds = _sha(pats, data)
+    assert hdr["patterns_sha256"] == ps and hdr["input_sha256"] == ds, "golden is for another workload"
+    prog = rx.Program(pats, **bench.PROGRAM_OPTS.get(config, {}))
+    dev = torch.device("cuda", 0)
+    d_in = torch.from_numpy(np.ascontiguousarray(data)).to(dev)
+    out = prog.alloc_outputs(nbytes, dev, dense=False, digests=True)
+    prog.match(d_in, out=out, stream=torch.cuda.current_stream(dev))
+    torch.cuda.synchronize()
+    counts = out["counts"].cpu().numpy().view(np.uint64)
+    digests = out["digests"].cpu().numpy().view(np.uint64)
+    assert int(out["status"].cpu()[0]) == 0
+    bad = np.nonzero((counts != g_counts) | (digests[:, 0] != g_d1) | (digests[:, 1] != g_d2))[0]
+    assert bad.size == 0, [(int(i), pats[i][:60], int(counts[i]), int(g_counts[i])) for i in bad[:8]]
+    assert int(g_counts.sum()) > 0
+    del d_in, out
+    torch.cuda.empty_cache()
+
+
 def test_snort_like_full_256mib_sampled():
     _check("snort", cap=64 << 20, prefix=6 << 20, windows=12, seed=21)
 

@@ -21,63 +21,126 @@ import oracle
 import paper_conf_micro_ge0025_b200 as rx
 
 
-def factors(prog):
-    """regex index -> list of factor byte strings (None: always runs)."""
-    out = {}
-    for line in prog.info.splitlines():
-        m = re.match(r"regex (\d+): factor (.*)", line)
-        if not m:
-            continue
-        i = int(m.group(1))
-        if m.group(2).startswith("none"):
-            out[i] = None
-            continue
-        grams = []
-        for tok in m.group(2).split("grams=")[1].strip(",").split(","):
-            h, k = tok.split("/")
-            g, k = int(h, 16), int(k)
-            grams.append(bytes((g >> (8 * (4 - k + j))) & 255 for j in range(k)))
-        out[i] = grams
+def _windows(toks):
+    """factor tokens "vvmm..vvmm@ae" -> [(values, masks, ae)]"""
+    out = []
+    for tok in toks:
+        body, ae = tok.split("@")
+        vals = bytes(int(body[i:i + 2], 16) for i in range(0, len(body), 4))
+        msks = bytes(int(body[i + 2:i + 4], 16) for i in range(0, len(body), 4))
+        out.append((vals, msks, int(ae.split("/")[0])))
     return out
 
 
+def factors(prog):
+    """regex index -> (first windows or None, output windows or None, delta)
+    from rx_program_info ("regex i: factor first W.. ; out W.. ; delta=D")."""
+    out = {}
+    for line in prog.info.splitlines():
+        m = re.match(r"regex (\d+): factor first (.*) ; out (.*) ; delta=(\d+)", line)
+        if not m:
+            continue
+        first = None if m.group(2).strip() == "none" else _windows(m.group(2).split())
+        outw = None if m.group(3).strip() == "none" else _windows(m.group(3).split())
+        out[int(m.group(1))] = (first, outw, int(m.group(4)))
+    return out
+
+
+def _occurrences(text, win):
+    """anchor-end positions e of the masked window (the window's bytes are
+    text[e - ae : e - ae + len]) lying wholly inside text"""
+    vals, msks, ae = win
+    n = len(vals)
+    hits = []
+    for st in range(0, len(text) - n + 1):
+        if all((text[st + j] & msks[j]) == vals[j] for j in range(n)):
+            hits.append((st, st + ae))
+    return hits
+
+
 HAND = [rb"abcd.*xyz", rb"(?:ab)+cdef", rb"wxyz[0-9]+q", rb"x(?:yz)*w", rb"(foo|ba[rz])", rb"q[^\n]*zz",
-        rb"ab[cd]{2}e", rb"(?:kk|ll)mmnn", rb"[ab]{3}c+", rb"hello(?:,? world)?!", rb"a.{0,5}bcd"]
+        rb"ab[cd]{2}e", rb"(?:kk|ll)mmnn", rb"[ab]{3}c+", rb"hello(?:,? world)?!", rb"a.{0,5}bcd",
+        rb"[a-z]+wxyz", rb"abc(?:de)*", rb"q[0-9]{2}(mn|kl)rs", rb"(?:xy|zw)+qq"]
+
+
+PLANTS = [b"abcdqqxyz", b"ababcdef", b"wxyz12q", b"xyzyzw", b"foo", b"bar", b"baz", b"q\nzz", b"qzz", b"abdce",
+          b"kkmmnn", b"llmmnn", b"hello, world!", b"hello!", b"a12bcd", b"abcdede", b"q12mnrs", b"q34klrs",
+          b"xyzwqq", b"zwxyqq", b"aabccc", b"kwxyz"]
 
 
 def test_factor_occurs_in_every_match_bruteforce():
+    # first factors: one lies inside every match (property (i)); output
+    # factors: one lies inside every match with its anchor end at most delta
+    # bytes before the match end (mode B) -- Python's re over all substrings
     rng = np.random.default_rng(5)
     pats = list(HAND)
-    while len(pats) < 60:
+    while len(pats) < 70:
         p = gen.fuzz_pattern(rng)
         if len(p) <= 20:
             pats.append(p)
     prog = rx.Program(pats)
     fac = factors(prog)
-    assert any(v is not None for v in fac.values())
-    alphabet = b"abcdefkl mnqrwxyz0123!,\n"
-    for _ in range(30):
-        n = int(rng.integers(5, 40))
-        text = bytes(alphabet[i] for i in rng.integers(0, len(alphabet), size=n))
+    assert sum(v[0] is not None for v in fac.values()) >= 10
+    assert sum(v[1] is not None for v in fac.values()) >= 10
+    alphabet = b"abcdefkl mnqrswxyz0123!,\n"
+    checked = {"first": 0, "out": 0}
+    for trial in range(40):
+        n = int(rng.integers(8, 40))
+        if trial % 2:
+            text = bytearray(gen.fuzz_text(rng, n))
+        else:
+            text = bytearray(alphabet[i] for i in rng.integers(0, len(alphabet), size=n))
+        for _ in range(2):
+            pl = PLANTS[int(rng.integers(0, len(PLANTS)))]
+            at = int(rng.integers(0, max(1, n - len(pl))))
+            text[at:at + len(pl)] = pl
+        text = bytes(text)
+        n = len(text)
         for i, p in enumerate(pats):
-            grams = fac[i]
-            if grams is None:
+            first, outw, delta = fac[i]
+            if first is None and outw is None:
                 continue
+            occ_f = [(st, len(w[0])) for w in (first or []) for (st, _) in _occurrences(text, w)]
+            occ_o = [(st, e, len(w[0])) for w in (outw or []) for (st, e) in _occurrences(text, w)]
             cre = re.compile(p)
             for s in range(n):
                 for e in range(s + 1, n + 1):
-                    if cre.fullmatch(text, s, e):
-                        sub = text[s:e]
-                        assert any(g in sub for g in grams), (p, sub, grams)
+                    if not cre.fullmatch(text, s, e):
+                        continue
+                    if first is not None:
+                        checked["first"] += 1
+                        assert any(s <= st and st + ln <= e for (st, ln) in occ_f), (p, text[s:e], first)
+                    if outw is not None:
+                        checked["out"] += 1
+                        assert any(s <= st and st + ln <= e and e - 1 - ae <= delta for (st, ae, ln) in occ_o), (
+                            p, text[s:e], outw, delta)
+    assert checked["first"] > 50 and checked["out"] > 50, checked
+
+
+def test_factor_windows_are_long_and_exact():
+    # extension windows: the whole fixed-offset literal prefix (<= 16 bytes),
+    # alternations of words branch, classes of one bit stay compared
+    prog = rx.Program([rb"HTTP/1\.union.+<script>", rb"GET(admin|root)xyz", rb"Cookie:[^\x00]*619ajavascript:",
+                       rb"[Ss]elect\s+from"])
+    fac = factors(prog)
+    (f0, o0, _), (f1, _, _), (f2, o2, d2), (f3, _, _) = fac[0], fac[1], fac[2], fac[3]
+    assert f0 is not None and bytes(v for v, m in zip(f0[0][0], f0[0][1]) if m == 0xff) == b"HTTP/1.union"
+    assert o0 is not None and bytes(v for v, m in zip(o0[0][0], o0[0][1]) if m == 0xff) == b"<script>"
+    assert sorted(bytes(w[0]) for w in f1) == [b"GETadminxyz", b"GETrootxyz"]
+    assert bytes(f2[0][0]) == b"Cookie:" and bytes(o2[0][0]) == b"619ajavascript:" and d2 <= 15
+    assert f3[0][1][0] == 0xdf and f3[0][0][1:6] == b"elect"   # [Ss] compared up to bit 5
 
 
 def test_stateful_factor_precedes_first_unbounded_repetition():
-    # property (ii): the factor is taken before the first unbounded repetition
-    prog = rx.Program([rb"(?:ab)+cdef", rb"xyzw[0-9]+qrst", rb"abcd.*wxyz"])
+    # property (ii): first factors are taken before the first unbounded
+    # repetition; output factors from the suffix after the last one
+    prog = rx.Program([rb"(?:ab)+cdef", rb"xyzw[0-9]+qrst", rb"abcd.*wxyz", rb"abcd[a-z]+"])
     fac = factors(prog)
-    assert fac[0] is None                      # nothing mandatory before (ab)+
-    assert all(g in b"xyzw" for g in fac[1])   # not "qrst"
-    assert all(g in b"abcd" for g in fac[2])   # not "wxyz"
+    assert fac[0][0] is None                           # nothing mandatory before (ab)+
+    assert bytes(fac[1][0][0][0]) == b"xyzw"           # not "qrst"
+    assert bytes(fac[2][0][0][0]) == b"abcd"           # not "wxyz"
+    assert bytes(fac[2][1][0][0]) == b"wxyz"           # output factor: the suffix
+    assert fac[3][1] is None                           # ends in a class-plus: no output factor
 
 
 gpu = pytest.mark.gpu
@@ -155,3 +218,57 @@ def test_snort_like_prefilter_vs_oracle(n):
     assert bad.size == 0, [(pats[i], int(g["counts"][i]), int(o["counts"][i])) for i in bad[:5]]
     assert np.array_equal(g["digests"], o["digests"])
     assert int(o["counts"].sum()) > 0
+
+
+def _modeb_input(rng, n, hot, rare, kill=b"\x00", kill_every=50000):
+    """text with a hot first factor every ~300 bytes, rare output factors
+    planted near 1 KiB-block and window edges, kill bytes now and then"""
+    alphabet = np.frombuffer(b"abcdefghijklmnopqrstuvwxyz0123456789 /=&.-", dtype=np.uint8)
+    buf = bytearray(alphabet[rng.integers(0, alphabet.size, size=n)].tobytes())
+    for at in range(int(rng.integers(0, 300)), n - 64, 300):
+        buf[at:at + len(hot)] = hot
+    spots = [int(x) for x in rng.integers(0, n - 64, size=12)] + [4093, 4095, 8190, 16383, 65535, 131070]
+    for at in spots:
+        if at + len(rare) < n:
+            buf[at:at + len(rare)] = rare
+    for at in range(kill_every // 2, n, kill_every):
+        buf[at:at + len(kill)] = kill
+    return bytes(buf)
+
+
+@gpu
+def test_mode_b_walk_back_bit_exact(capfd):
+    # hot first factors ("Cookie:", "HTTP/1.") with rare output factors: the
+    # clusters run output-gated (mode B) and reconstruct their incoming state
+    # by walking back -- across long [^\x00]* carries, while-loop frontiers,
+    # segment boundaries and up to the stream start
+    pats = [rb"Cookie:[^\x00]*619ajavascript:", rb"HTTP/1\.(?:%[0-9a-f]{2})*DpPXrWa(?:iJ4/)*",
+            rb"Cookie:[a-z]+=qz7Kx", rb"HTTP/1\.[^\r\n]*q9Zz", rb"zz[0-9]+", rb"abc"]
+    rng = np.random.default_rng(3)
+    prog = rx.Program(pats, flags=rx.RX_F_STATS)
+    plants = [b"619ajavascript:", b"%2f%3aDpPXrWaiJ4/iJ4/", b"DpPXrWa", b"abc=qz7Kx", b"q9Zz"]
+    for n in (5000, 200000, (3 << 20) + 123):
+        a = _modeb_input(rng, n, b"Cookie:", plants[0])
+        b = _modeb_input(rng, n, b"HTTP/1.", plants[int(rng.integers(1, len(plants)))], kill=b"\r\n")
+        # alternate 3 KiB pieces of the two texts
+        data = b"".join((a if (i // 3072) % 2 else b)[i:i + 3072] for i in range(0, n, 3072))[:n]
+        data = data[: n // 3] + b"Cookie:abc=qz7KxHTTP/1.%2fDpPXrWaiJ4/" + data[n // 3:]
+        g = _gpu_counts(prog, data, dense=True)
+        o = oracle.run_set(pats, data, dense=True)
+        assert g["status"] == 0
+        assert np.array_equal(g["counts"], o["counts"]), (n, g["counts"], o["counts"])
+        assert np.array_equal(g["digests"], o["digests"])
+        assert np.array_equal(g["dense"], o["dense"][:, : g["dense"].shape[1]])
+    err = capfd.readouterr().err
+    assert "modeB_members=" in err and re.search(r"modeB_members=[1-9]", err), err[-2000:]
+    assert re.search(r"walkbacks=[1-9]", err), err[-2000:]
+
+
+@gpu
+def test_mode_b_off_equals_on():
+    # the ablation flag (RX_F_NO_MODEB) gives the same result on the Snort-like set
+    pats = gen.snort_patterns(300, 2)[0]
+    data = bytes(gen.snort_input((1 << 20) + 5, seed=7))
+    a = _gpu_counts(rx.Program(pats), data)
+    b = _gpu_counts(rx.Program(pats, flags=rx.RX_F_NO_MODEB), data)
+    assert np.array_equal(a["counts"], b["counts"]) and np.array_equal(a["digests"], b["digests"])
