@@ -235,6 +235,8 @@ def main():
     ap.add_argument("--no-prefilter", action="store_true", help="ablation: RX_F_NO_PREFILTER")
     ap.add_argument("--words-per-lane", type=int, default=0, help="experiment: minimum K (rx_options.words_per_lane)")
     ap.add_argument("--group-size", type=int, default=0, help="experiment: max regexes per group (rx_options)")
+    ap.add_argument("--ablate", default="", help="comma list of rx flags to set (ablation ladder, DESIGN.md): "
+                    "no_prefilter, no_modeb, no_lockstep, no_guards, rebalance")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -259,7 +261,10 @@ def main():
         popts["words_per_lane"] = args.words_per_lane
     if args.group_size:
         popts["group_size"] = args.group_size
-    prog = rx.Program(pats, flags=rx.RX_F_NO_PREFILTER if args.no_prefilter else 0, **popts)
+    flags = rx.RX_F_NO_PREFILTER if args.no_prefilter else 0
+    for a in filter(None, args.ablate.split(",")):
+        flags |= getattr(rx, "RX_F_" + a.upper())
+    prog = rx.Program(pats, flags=flags, **popts)
     compile_s = time.perf_counter() - t0
 
     host = torch.from_numpy(np.ascontiguousarray(data)).pin_memory()
@@ -350,7 +355,7 @@ def main():
                    "groups": prog.n_groups, "outputs": "per-regex counts (dense streams off: 31 GiB at this size)",
                    "l2": f"input {nbytes >> 20} MiB per GPU" + (" > 126 MB L2: no flush needed" if nbytes > (126 << 20)
                                                                   else " < L2: L2 flushed between steps"),
-                   "prefilter": not args.no_prefilter, "compile_s": round(compile_s, 1),
+                   "prefilter": not args.no_prefilter, "ablate": args.ablate or None, "compile_s": round(compile_s, 1),
                    **popts},
         "roofline": roofline(ktimes, nbytes, len(pats), hbm, hbm_src, name, ms),
         "clocks": clocks,

@@ -78,6 +78,8 @@ typedef struct {
                                  runs every window, gated only by Zero Block Skipping (Sec. 6) */
 #define RX_F_NO_MODEB 32u     /* never run a cluster output-gated: with the prefilter on, a
                                  cluster runs where its first factor occurs or state flows in (ablation) */
+#define RX_F_NO_LOCKSTEP 128u /* sparse pass 1 without cluster lockstep: each warp runs its own windows'
+                                 clusters freely (ablation) */
 #define RX_F_STATS 64u        /* debug: count visited / active windows and walk-backs per rx_match and print
                                  them to stderr (synchronises the stream; not for timing) */
 

@@ -304,6 +304,7 @@ struct RxParams {
   int mode;                 // 0 = pass 1, 1 = fix-up with stored segment states, 2 = rematch
   int accumulate;           // counts/digests are added to (else the host zeroed them)
   int modeb;                // mode B allowed (plain rx_match: no chunk state in/out)
+  int lockstep;             // sparse pass 1: cluster lockstep across the CTA's warps (rx_run_segment_pf)
   // cross-regex prefilter (rx_prefilter_run below; rx_prefilter.cpp
   // build_prefilter documents the table blob)
   const u32 *pf_tab;
@@ -797,63 +798,114 @@ DEV void rx_run_segment_pf(const RxParams &p, int seg, RxOut *o, u64 *acc, u32 *
   u32 exact = 0u;  // mode-B clusters whose state in st[] is exact at window w
   i64 w = pending_a(st) ? w_begin : next_hit(w_begin);
   if (w < w_end) stage(w);
-  while (w < w_end) {
-    const u32 pendc = NS > 0 ? rx_pend_clusters<G>(st, c.lane) : 0u;
-    const bool pend_in = (pendc & ~bmc) != 0u;
-    if (p.stats && c.lane == 0) atomicAdd(&p.stats[3], 1ull);
-    i64 b0, b1;
-    frame_blocks(w, b0, b1);
-    u32 fmine = 0u, omine = 0u;
-    for (i64 b = b0 + c.lane; b <= b1; b += 32)
-      if ((gb[b >> 5] >> (b & 31)) & 1u) {
-        fmine |= mmf[b];
-        omine |= mmo[b];
+  // Cluster lockstep (p.lockstep): the CTA's
+  // warps (one group, 16 segments) take one window each per round and then
+  // walk the union of their cluster masks in ascending order with one CTA
+  // barrier per cluster, so the warps that run a cluster run it together and
+  // the SM fetches its straight-line code once for all of them (the
+  // instruction-fetch stall, no_instructions, was the top stall of the
+  // free-running form: profiles/r2_ncu_*).  Windows with nothing to run are
+  // skipped between rounds without a barrier.
+  __shared__ u32 rx_cta_union[2];
+  const bool lock = p.lockstep != 0;
+  int par = 0;
+  if (lock) {
+    if (threadIdx.x == 0) rx_cta_union[0] = rx_cta_union[1] = 0u;
+    __syncthreads();
+  }
+  for (;;) {
+    // the next window with something to run (w_end: none left)
+    u32 run = 0u, pendc = 0u;
+    bool pend_in = false;
+    while (w < w_end) {
+      pendc = NS > 0 ? rx_pend_clusters<G>(st, c.lane) : 0u;
+      pend_in = (pendc & ~bmc) != 0u;
+      if (p.stats && c.lane == 0) atomicAdd(&p.stats[3], 1ull);
+      i64 b0, b1;
+      frame_blocks(w, b0, b1);
+      u32 fmine = 0u, omine = 0u;
+      for (i64 b = b0 + c.lane; b <= b1; b += 32)
+        if ((gb[b >> 5] >> (b & 31)) & 1u) {
+          fmine |= mmf[b];
+          omine |= mmo[b];
+        }
+      const u32 fm = __reduce_or_sync(RX_FULL, fmine), om = __reduce_or_sync(RX_FULL, omine);
+      const u32 rmask = (fm & ~bm) | (om & bm);
+      if (rmask == 0u && !pend_in && always_a == 0u) {
+        exact = 0u;
+        w = next_hit(w + 1);
+        continue;
       }
-    const u32 fm = __reduce_or_sync(RX_FULL, fmine), om = __reduce_or_sync(RX_FULL, omine);
-    const u32 rmask = (fm & ~bm) | (om & bm);
-    if (rmask == 0u && !pend_in && always_a == 0u) {
-      exact = 0u;
-      w = next_hit(w + 1);
-      continue;
+      // the clusters to run (never empty here: a hit, carried state or a
+      // member without a factor each select a cluster)
+      run = rx_run_clusters<G>(rmask, bmc, pendc, c.lane);
+      if (p.stats && c.lane == 0) {
+        atomicAdd(&p.stats[0], 1ull);
+        atomicAdd(&p.stats[2], (u64)__popc(rmask));
+        atomicAdd(&p.stats[6], (u64)__popc(run));
+        u64 *gs = p.stats + 8 + 4 * G::GID;  // per group: active windows, member hits, mode-B clusters, cluster runs
+        atomicAdd(&gs[0], 1ull);
+        atomicAdd(&gs[1], (u64)__popc(rmask));
+        gs[2] = (u64)__popc(bmc);
+        atomicAdd(&gs[3], (u64)__popc(run));
+      }
+      break;
     }
-    // the clusters to run; those of them in mode B whose state is stale
-    // first reconstruct it
-    const u32 run = rx_run_clusters<G>(rmask, bmc, pendc, c.lane);
+    const bool have = w < w_end;
     const u32 runb = run & bmc;
-    const u32 stale = runb & ~exact;
-    if (stale) rx_walk_back<G>(p, ir, c, pl, xr, w, stale, st, wbs, len_words);
-    const i64 fword = w * Bw - Lw;
-    if (staged == w) {
-      retire();
-      const uint4 *q = reinterpret_cast<const uint4 *>(tbuf + c.lane * (32u * K));
+    if (have) {
+      // mode-B clusters to run whose state is stale first reconstruct it
+      const u32 stale = runb & ~exact;
+      if (stale) rx_walk_back<G>(p, ir, c, pl, xr, w, stale, st, wbs, len_words);
+      const i64 fword = w * Bw - Lw;
+      if (staged == w) {
+        retire();
+        const uint4 *q = reinterpret_cast<const uint4 *>(tbuf + c.lane * (32u * K));
 #pragma unroll
-      for (int k = 0; k < K; ++k) {
-        const uint4 a0 = q[2 * k], a1 = q[2 * k + 1];
-        xr[k][0] = a0.x; xr[k][1] = a0.y; xr[k][2] = a0.z; xr[k][3] = a0.w;
-        xr[k][4] = a1.x; xr[k][5] = a1.y; xr[k][6] = a1.z; xr[k][7] = a1.w;
+        for (int k = 0; k < K; ++k) {
+          const uint4 a0 = q[2 * k], a1 = q[2 * k + 1];
+          xr[k][0] = a0.x; xr[k][1] = a0.y; xr[k][2] = a0.z; xr[k][3] = a0.w;
+          xr[k][4] = a1.x; xr[k][5] = a1.y; xr[k][6] = a1.z; xr[k][7] = a1.w;
+        }
+      } else {
+        if (staged >= 0) retire();  // a stale guess: drain it
+        rx_fetch<K>(p, ir, c.lane, xr, fword);
       }
-    } else {
-      if (staged >= 0) retire();  // a stale guess: drain it
-      rx_fetch<K>(p, ir, c.lane, xr, fword);
+      // guess the next window and start its copy before the body runs
+      if (staged < 0) stage(pend_in ? w + 1 : next_hit(w + 1));
+      c.cw = (u32)((len_words - w * Bw) < Bw ? (len_words - w * Bw) : Bw);
+      c.word0 = fword;
+      rx_unpack<K>(p, ir, c, xr, pl, fword);
+      rx_commit_mask(p, ir, c, Lw, fword);
+      if (NS > 0) rx_state_zero(nst, NS, c.lane);
     }
-    // guess the next window and start its copy before the body runs
-    if (staged < 0) stage(pend_in ? w + 1 : next_hit(w + 1));
-    if (p.stats && c.lane == 0) {
-      atomicAdd(&p.stats[0], 1ull);
-      atomicAdd(&p.stats[2], (u64)__popc(rmask));
-      atomicAdd(&p.stats[6], (u64)__popc(run));
-      u64 *gs = p.stats + 8 + 4 * G::GID;  // per group: active windows, member hits, mode-B clusters, cluster runs
-      atomicAdd(&gs[0], 1ull);
-      atomicAdd(&gs[1], (u64)__popc(rmask));
-      gs[2] = (u64)__popc(bmc);
-      atomicAdd(&gs[3], (u64)__popc(run));
+    // the clusters this round walks: the CTA's union (lockstep) or this
+    // warp's own mask; one call site of the inlined body either way
+    u32 U = run;
+    if (lock) {
+      if (have && c.lane == 0) atomicOr(&rx_cta_union[par], run);
+      const int more = __syncthreads_or(have);
+      U = rx_cta_union[par];
+      // every warp read the other word before this round's barrier
+      if (threadIdx.x == 0) rx_cta_union[par ^ 1] = 0u;
+      par ^= 1;
+      if (!more) break;
+    } else if (!have) {
+      break;
     }
-    c.cw = (u32)((len_words - w * Bw) < Bw ? (len_words - w * Bw) : Bw);
-    c.word0 = fword;
-    rx_unpack<K>(p, ir, c, xr, pl, fword);
-    rx_commit_mask(p, ir, c, Lw, fword);
-    if (NS > 0) rx_state_zero(nst, NS, c.lane);
-    G::body_i(c, pl, st, nst, run);
+    while (U) {
+      u32 m = run;
+      if (lock) {
+        const u32 bit = U & (0u - U);
+        U &= U - 1u;
+        m = run & bit;
+      } else {
+        U = 0u;
+      }
+      if (m) G::body_i(c, pl, st, nst, m);
+      if (lock) __syncthreads();
+    }
+    if (!have) continue;
     u32 *t = st;
     st = nst;
     nst = t;

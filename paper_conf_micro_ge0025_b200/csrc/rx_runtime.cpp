@@ -564,6 +564,7 @@ struct RxParamsHost {  // must mirror RxParams in rx_device.cuh (tests/test_libr
   int mode;
   int accumulate;
   int modeb;
+  int lockstep;
   const unsigned int *pf_tab;
   unsigned int pf_words, pf_smem_words;
   unsigned int pf_b4bits, pf_b3bits, pf_hbits;
@@ -722,6 +723,7 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
   // stream: its walk-back may read any earlier byte and reconstructs state
   // from the stream start, so chunks (incoming / outgoing state) use mode A
   prm.modeb = (mode == 0 && !st_in && !st_out && halo_left == 0) ? 1 : 0;
+  prm.lockstep = (p->flags & RX_F_NO_LOCKSTEP) ? 0 : 1;
   if (!prm.status) {
     unsigned int *status_scratch = (unsigned int *)scratch_get(p, stream, SC_STATUS, 256);
     if (!status_scratch) return fail(RX_ENOMEM, "status");
