@@ -11,10 +11,18 @@ payloads (BASELINE.json configs[1]).
   python bench.py [--gpus N] [--steps K] [--warmup W] [--config snort|tiny|...]
   python bench.py --impl reference ...   # the CPU oracle, timed on a bounded sample
 
-Multi-GPU (torchrun, one rank per GPU, NCCL): weak scaling by input chunks --
-rank r scans its own 256 MiB chunk of one N x 256 MiB stream (halo bytes from
-the neighbour chunk, boundary state exchanged with all_gather, carry fix-up
-with rx_rematch_chunk, counts all-reduced).
+Multi-GPU (torchrun, one rank per GPU, NCCL), DESIGN.md "Multi-GPU":
+  --split chunk (default, weak scaling): the stream is N x 256 MiB; rank r
+    holds chunk r (generated with its own seed) at global offset r x 256 MiB.
+    Every timed step exchanges the halos (rx_max_lookback / lookahead bytes of
+    the neighbour chunks, one all_gather), matches the chunk speculatively,
+    resolves the boundary states (all_gather rounds + rx_rematch_chunk where
+    a rank's true incoming state differs) and all-reduces the counts, so
+    every rank ends with the whole stream's exact counts
+    (paper_conf_micro_ge0025_b200/parallel.py).
+  --split regex (strong scaling): rank r compiles its share of the regex set
+    (parallel.shard_patterns) and scans the same input; each step scatters
+    its counts into the full per-regex vector and all-reduces it.
 
 Timing: CUDA events on the matching stream around exactly K steps, barrier +
 synchronize on both sides, max over ranks.  The input (256 MiB) is larger
@@ -235,8 +243,12 @@ def main():
     ap.add_argument("--no-prefilter", action="store_true", help="ablation: RX_F_NO_PREFILTER")
     ap.add_argument("--words-per-lane", type=int, default=0, help="experiment: minimum K (rx_options.words_per_lane)")
     ap.add_argument("--group-size", type=int, default=0, help="experiment: max regexes per group (rx_options)")
+    ap.add_argument("--max-regs", type=int, default=0, help="experiment: registers per thread (rx_options; "
+                    "pass-1 CTA = 64K / (32 x max_regs) warps)")
+    ap.add_argument("--interval", type=int, default=0, help="experiment: zero-block guard interval (rx_options)")
+    ap.add_argument("--split", default="chunk", choices=["chunk", "regex"], help="multi-GPU partition (N>1)")
     ap.add_argument("--ablate", default="", help="comma list of rx flags to set (ablation ladder, DESIGN.md): "
-                    "no_prefilter, no_modeb, no_lockstep, no_guards, rebalance")
+                    "no_prefilter, modeb, no_lockstep, no_guards, rebalance")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -253,14 +265,27 @@ def main():
     dev = torch.device("cuda", local)
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
-    pats, data, nbytes, name = load_workload(args.config, (args.length_mib << 20) if args.length_mib else None, rank)
+    split_regex = world > 1 and args.split == "regex"
+    # regex split: every rank scans the same input (rank 0's); chunk split:
+    # rank r's own chunk of the stream
+    pats, data, nbytes, name = load_workload(args.config, (args.length_mib << 20) if args.length_mib else None,
+                                             0 if split_regex else rank)
     nbytes = int(data.size)
+    all_pats = pats
+    if split_regex:
+        from paper_conf_micro_ge0025_b200 import parallel
+        mine = parallel.shard_patterns(len(pats), world, rank, costs=[float(len(p)) for p in pats])
+        pats = [pats[i] for i in mine]
     t0 = time.perf_counter()
     popts = dict(PROGRAM_OPTS.get(args.config, {}))
     if args.words_per_lane:
         popts["words_per_lane"] = args.words_per_lane
     if args.group_size:
         popts["group_size"] = args.group_size
+    if args.interval:
+        popts["interval"] = args.interval
+    if args.max_regs:
+        popts["max_regs"] = args.max_regs
     flags = rx.RX_F_NO_PREFILTER if args.no_prefilter else 0
     for a in filter(None, args.ablate.split(",")):
         flags |= getattr(rx, "RX_F_" + a.upper())
@@ -276,16 +301,27 @@ def main():
         prog.match(d_in, out=out, stream=stream)
 
     def step_e2e():
+        # the public API end to end: H2D of the step's input from pinned host
+        # memory, the step (with its collectives at N > 1), D2H of the counts
         d_in.copy_(host, non_blocking=True)
-        prog.match(d_in, out=out, stream=stream)
-        return out["counts"].to("cpu", non_blocking=False)
+        step_device()
+        return (full if split_regex else out["counts"]).to("cpu", non_blocking=False)
 
-    if world > 1:
+    if world > 1 and not split_regex:
         from paper_conf_micro_ge0025_b200 import parallel
         ctx = parallel.ChunkMatcher(prog, dev)
 
         def step_device():  # noqa: F811
-            ctx.match_stream_chunk(d_in, rank, world, out)
+            ctx.match_stream_chunk(d_in, rank, world, out, rank * nbytes)
+    elif split_regex:
+        full = torch.zeros(len(all_pats), dtype=torch.int64, device=dev)
+        idx = torch.tensor(mine, dtype=torch.int64, device=dev)
+
+        def step_device():  # noqa: F811
+            prog.match(d_in, out=out, stream=stream)
+            full.zero_()
+            full.index_copy_(0, idx, out["counts"])
+            dist.all_reduce(full)
 
     for _ in range(args.warmup):
         step_device()
@@ -341,17 +377,19 @@ def main():
     prog.set_profiling(False)
     # e2e through the public API with host buffers (H2D of the step's input,
     # D2H of the counts) -- same metric
-    e2e_ms = timed(step_e2e, max(1, min(args.steps, 5))) if world == 1 else None
+    e2e_ms = timed(step_e2e, max(1, min(args.steps, 5)))
 
-    total_bytes = nbytes * world
+    total_bytes = nbytes if split_regex else nbytes * world
     gbs = total_bytes / (ms * 1e-3) / 1e9
     hbm, hbm_src = measured_peaks()
     launches_per_step = prog.kernels_per_match
     line = {
         "metric": "input GB/s scanned per regex set", "value": gbs, "unit": "GB/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
-        "config": {"workload": name, "n_regex": len(pats), "input_bytes_per_gpu": nbytes,
+        "scaling": "strong" if split_regex else "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+        "config": {"workload": name, "n_regex": len(all_pats), "input_bytes_per_gpu": nbytes,
+                   "parallelism": (f"regex-shard x{world}" if split_regex else f"input-chunk x{world}") if world > 1
+                   else "1 GPU",
                    "groups": prog.n_groups, "outputs": "per-regex counts (dense streams off: 31 GiB at this size)",
                    "l2": f"input {nbytes >> 20} MiB per GPU" + (" > 126 MB L2: no flush needed" if nbytes > (126 << 20)
                                                                   else " < L2: L2 flushed between steps"),
@@ -362,8 +400,8 @@ def main():
         "gpu_launches": sum(v[1] for v in ktimes.values()) or launches_per_step * args.steps,
     }
     if e2e_ms is not None:
-        line["e2e"] = {"value": nbytes / (e2e_ms * 1e-3) / 1e9, "unit": "GB/s", "h2d_bytes_per_step": nbytes,
-                       "d2h_bytes_per_step": 8 * len(pats)}
+        line["e2e"] = {"value": total_bytes / (e2e_ms * 1e-3) / 1e9, "unit": "GB/s", "h2d_bytes_per_step": nbytes,
+                       "d2h_bytes_per_step": 8 * len(all_pats)}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         r, n, dt, thr = oracle_rate(pats, data, target_s=15.0)
         line["cpu_baseline"] = {"value": r, "unit": "GB/s", "cores": thr, "kind": "oracle",

@@ -60,7 +60,7 @@ typedef struct {
 /* Tunables.  Defaults follow the paper's fixed defaults (merge size 8,
  * interval size 8, CTA count 256, max registers 128) where they apply. */
 typedef struct {
-  uint32_t interval;       /* zero-block-skipping guard interval in IR instructions (Sec. 6); 0 = default 8; UINT32_MAX = no guards */
+  uint32_t interval;       /* zero-block-skipping guard interval in IR instructions (Sec. 6); 0 = default 4 (the paper: 8); UINT32_MAX = no guards */
   uint32_t max_regs;       /* NVRTC --maxrregcount; 0 = default 128 */
   uint32_t group_size;     /* max regexes per group; 0 = auto */
   uint32_t words_per_lane; /* K: 32-bit words per lane per window (window = 1024*K positions): 0 (auto), 1, 2, 4
@@ -76,8 +76,11 @@ typedef struct {
 #define RX_F_NO_CACHE 4u     /* do not read/write the on-disk cubin cache */
 #define RX_F_NO_PREFILTER 16u /* disable the cross-regex literal prefilter: every group
                                  runs every window, gated only by Zero Block Skipping (Sec. 6) */
-#define RX_F_NO_MODEB 32u     /* never run a cluster output-gated: with the prefilter on, a
-                                 cluster runs where its first factor occurs or state flows in (ablation) */
+#define RX_F_NO_MODEB 32u     /* accepted for compatibility: mode B is off unless RX_F_MODEB */
+#define RX_F_MODEB 256u       /* allow output-gated clusters: a cluster whose members all have
+                                 output factors may run only where one occurs, reconstructing its incoming state by a
+                                 walk-back.  Off by default: measured slower on the Snort-like set (ablation ladder,
+                                 profiles/r2_ablation_snort.md) */
 #define RX_F_NO_LOCKSTEP 128u /* sparse pass 1 without cluster lockstep: each warp runs its own windows'
                                  clusters freely (ablation) */
 #define RX_F_STATS 64u        /* debug: count visited / active windows and walk-backs per rx_match and print

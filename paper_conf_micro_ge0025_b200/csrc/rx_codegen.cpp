@@ -625,10 +625,14 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
   const int PER = ACC + OUTB + STB + LB + TB + 16;
   os << "static_assert(sizeof(RxOut) <= " << OUTB << ", \"RxOut layout\");\n";
   os << "#define RX_WARP_SMEM_" << gi << " " << PER << "\n";
-  os << "extern \"C\" __device__ __noinline__ void rx_seg_" << gi << "(const RxParams &p, int seg) {\n"
-     << "  extern __shared__ __align__(16) u64 rx_smem[];\n"
+  // The launch parameters are read from the CTA header of the dynamic shared
+  // memory (rx_cta_params, copied there by the kernel): a reference to the
+  // kernel parameter handed across this out-of-line call made every field
+  // read a generic load through a spilled pointer (profiles/r2_*).
+  os << "extern \"C\" __device__ __noinline__ void rx_seg_" << gi << "(int seg) {\n"
+     << "  const RxParams &p = rx_cta_params();\n"
      << "  const int warp = threadIdx.x >> 5;\n"
-     << "  unsigned char *base = reinterpret_cast<unsigned char *>(rx_smem) + (size_t)warp * " << PER << ";\n"
+     << "  unsigned char *base = rx_warp_smem(warp, " << PER << ");\n"
      << "  u64 *acc = reinterpret_cast<u64 *>(base);\n"
      << "  RxOut *o = reinterpret_cast<RxOut *>(base + " << ACC << ");\n"
      << "  u32 *st = reinterpret_cast<u32 *>(base + " << ACC + OUTB << ");\n"
@@ -640,10 +644,10 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
     os << "  if (p.pf_on) { rx_run_segment_pf<RxG" << gi << ">(p, seg, o, acc, st, tb, bar, lb); return; }\n";
   os << "  rx_run_segment_dense<RxG" << gi << ">(p, seg, o, acc, st, lb);\n}\n";
   if (g.nslots > 0)
-    os << "extern \"C\" __device__ __noinline__ void rx_fix_" << gi << "(const RxParams &p, int seg) {\n"
-       << "  extern __shared__ __align__(16) u64 rx_smem[];\n"
+    os << "extern \"C\" __device__ __noinline__ void rx_fix_" << gi << "(int seg) {\n"
+       << "  const RxParams &p = rx_cta_params();\n"
        << "  const int warp = threadIdx.x >> 5;\n"
-       << "  unsigned char *base = reinterpret_cast<unsigned char *>(rx_smem) + (size_t)warp * " << PER << ";\n"
+       << "  unsigned char *base = rx_warp_smem(warp, " << PER << ");\n"
        << "  rx_fixup_group<RxG" << gi << ">(p, reinterpret_cast<RxOut *>(base + " << ACC
        << "), reinterpret_cast<u64 *>(base), reinterpret_cast<u32 *>(base + " << ACC + OUTB << "), base + "
        << ACC + OUTB + STB << ", seg);\n}\n";
@@ -661,24 +665,26 @@ size_t warp_smem_bytes(const CompiledSet &cs) {
 // The kernel unit: rx_pass1 (a CTA of 16 warps runs one group over 16
 // consecutive segments), rx_prefilter, rx_fixup (phase 1: one warp per
 // (group, segment); phase 2 and rematch: one warp per group).
-std::string emit_kernel_unit(CompiledSet &cs) {
+std::string emit_kernel_unit(CompiledSet &cs, int gb, int ge) {
   std::ostringstream os;
-  os << kDevicePrelude << "\n// ===================== kernels =====================\n";
+  os << kDevicePrelude << "\n// ===================== kernels (groups " << gb << ".." << ge - 1
+     << ") =====================\n";
   int G = (int)cs.groups.size();
-  os << "#define RX_NG " << G << "\n";
-  for (int gi = 0; gi < G; ++gi) {
-    os << "extern \"C\" __device__ void rx_seg_" << gi << "(const RxParams &p, int seg);\n";
-    if (cs.groups[gi].nslots > 0) os << "extern \"C\" __device__ void rx_fix_" << gi << "(const RxParams &p, int seg);\n";
+  os << "#define RX_NG " << G << "\n#define RX_G0 " << gb << "\n#define RX_G1 " << ge << "\n";
+  for (int gi = gb; gi < ge; ++gi) {
+    os << "extern \"C\" __device__ void rx_seg_" << gi << "(int seg);\n";
+    if (cs.groups[gi].nslots > 0) os << "extern \"C\" __device__ void rx_fix_" << gi << "(int seg);\n";
   }
-  os << "\nextern \"C\" __global__ void __launch_bounds__(512, 1) rx_pass1(const RxParams p) {\n"
+  os << "\nextern \"C\" __global__ void __launch_bounds__(" << 32 * cs.pass1_warps << ", 1) rx_pass1(const RxParams p) {\n"
         "  const int warp = threadIdx.x >> 5;\n"
         "  const int wpb = blockDim.x >> 5;\n"
         "  const int cpg = (p.nseg_max + wpb - 1) / wpb;  // CTAs per group\n"
-        "  const int g = (int)(blockIdx.x / cpg);\n"
+        "  const int g = RX_G0 + (int)(blockIdx.x / cpg);\n"
         "  const long long seg = (long long)(blockIdx.x % cpg) * wpb + warp;\n"
-        "  if (g >= RX_NG) return;\n"
+        "  if (g >= RX_G1) return;\n"
+        "  rx_cta_params_store(p);\n"
         "  switch (g) {\n";
-  for (int gi = 0; gi < G; ++gi) os << "    case " << gi << ": rx_seg_" << gi << "(p, (int)seg); break;\n";
+  for (int gi = gb; gi < ge; ++gi) os << "    case " << gi << ": rx_seg_" << gi << "((int)seg); break;\n";
   os << "    default: break;\n  }\n}\n";
   if (cs.use_pf)
     os << "\nextern \"C\" __global__ void __launch_bounds__(256, 3) rx_prefilter(const RxParams p) {\n"
@@ -688,12 +694,13 @@ std::string emit_kernel_unit(CompiledSet &cs) {
         "  const int wpb = blockDim.x >> 5;\n"
         "  const long long gw = (long long)blockIdx.x * wpb + warp;\n"
         "  // phase 1: warp -> (group, segment); otherwise warp -> group\n"
-        "  const long long g = p.fix_phase == 1 ? gw / p.nseg_max : gw;\n"
+        "  const long long g = RX_G0 + (p.fix_phase == 1 ? gw / p.nseg_max : gw);\n"
         "  const int seg = p.fix_phase == 1 ? (int)(gw % p.nseg_max) : 0;\n"
-        "  if (g >= RX_NG) return;\n"
+        "  rx_cta_params_store(p);\n"
+        "  if (g >= RX_G1) return;\n"
         "  switch ((int)g) {\n";
-  for (int gi = 0; gi < G; ++gi)
-    if (cs.groups[gi].nslots > 0) os << "    case " << gi << ": rx_fix_" << gi << "(p, seg); break;\n";
+  for (int gi = gb; gi < ge; ++gi)
+    if (cs.groups[gi].nslots > 0) os << "    case " << gi << ": rx_fix_" << gi << "(seg); break;\n";
   os << "    default: break;\n  }\n}\n";
   return os.str();
 }

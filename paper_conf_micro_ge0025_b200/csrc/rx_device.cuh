@@ -327,6 +327,25 @@ struct RxParams {
   u32 *seg_nc;              // [nseg_max][G]: that segment did not converge in phase 1
 };
 
+// CTA header of the dynamic shared memory (pass 1 and fix-up): the launch
+// parameters (copied once per CTA by the kernel, then read with LDS at fixed
+// offsets) and the cluster-lockstep union words; the per-warp areas follow.
+#define RX_CTA_HDR 512
+static_assert(sizeof(RxParams) <= 496, "RxParams must fit the CTA header");
+DEV unsigned char *rx_dyn_smem() {
+  extern __shared__ __align__(16) u64 rx_smem[];
+  return reinterpret_cast<unsigned char *>(rx_smem);
+}
+DEV const RxParams &rx_cta_params() { return *reinterpret_cast<const RxParams *>(rx_dyn_smem()); }
+DEV u32 *rx_cta_union() { return reinterpret_cast<u32 *>(rx_dyn_smem() + 496); }
+DEV unsigned char *rx_warp_smem(int warp, int per) { return rx_dyn_smem() + RX_CTA_HDR + (size_t)warp * per; }
+DEV void rx_cta_params_store(const RxParams &p) {
+  const u32 *src = reinterpret_cast<const u32 *>(&p);
+  u32 *dst = reinterpret_cast<u32 *>(rx_dyn_smem());
+  for (int i = threadIdx.x; i < (int)(sizeof(RxParams) / 4); i += blockDim.x) dst[i] = src[i];
+  __syncthreads();
+}
+
 // split prologue (software pipelining): rx_fetch issues the 128-bit loads of
 // a window into registers, rx_unpack transposes them.  Interior windows (all
 // bytes readable and valid, 16-byte aligned) take the straight path; edge
@@ -646,11 +665,18 @@ template <class G> DEV bool rx_state_eq_cl(const u32 *a, const u32 *b, u32 cl, u
 // once both runs agree, that is the true state.  d doubles until they agree
 // or the walk reaches the stream start (state zero).  Runs are state-only
 // (c.walk: no output) and execute only the stale clusters.
+//
+// The walk-back has its own window context and planes: they are handed to
+// the out-of-line body by reference, and sharing the runner's would force
+// the runner's copies into local memory for the whole segment loop.
 template <class G>
-DEV void rx_walk_back(const RxParams &p, const RxRange &ir, Ctx<G::K> &c, u32 (&pl)[8][G::K], u32 (&xr)[G::K][8],
-                      i64 w, u32 stale, u32 *st, u32 *wb, i64 len_words) {
+__device__ __noinline__ void rx_walk_back(const RxParams &p, const RxRange &ir, const Ctx<G::K> cin, i64 w, u32 stale,
+                                          u32 *st, u32 *wb, i64 len_words) {
   constexpr int K = G::K, Lw = G::Lw, Bw = G::Bw, NS = G::NS, M = G::NSMAX;
   u32 *s0 = wb, *n0 = wb + M, *s1 = wb + 2 * M, *n1 = wb + 3 * M;
+  Ctx<K> c = cin;
+  u32 pl[8][K];
+  u32 xr[K][8];
   c.walk = true;
   int rounds = 0;
   for (i64 d = 1;; d *= 2) {
@@ -689,7 +715,6 @@ DEV void rx_walk_back(const RxParams &p, const RxRange &ir, Ctx<G::K> &c, u32 (&
   for (int s = (int)c.lane; s < NS; s += 32)
     if ((stale >> G::sci(s)) & 1u) st[s] = s0[s];
   __syncwarp();
-  c.walk = false;
   if (p.stats && c.lane == 0) {
     atomicAdd(&p.stats[4], 1ull);
     atomicAdd(&p.stats[5], (u64)rounds);
@@ -806,11 +831,11 @@ DEV void rx_run_segment_pf(const RxParams &p, int seg, RxOut *o, u64 *acc, u32 *
   // instruction-fetch stall, no_instructions, was the top stall of the
   // free-running form: profiles/r2_ncu_*).  Windows with nothing to run are
   // skipped between rounds without a barrier.
-  __shared__ u32 rx_cta_union[2];
+  u32 *const rx_cta_u = rx_cta_union();
   const bool lock = p.lockstep != 0;
   int par = 0;
   if (lock) {
-    if (threadIdx.x == 0) rx_cta_union[0] = rx_cta_union[1] = 0u;
+    if (threadIdx.x == 0) rx_cta_u[0] = rx_cta_u[1] = 0u;
     __syncthreads();
   }
   for (;;) {
@@ -856,7 +881,7 @@ DEV void rx_run_segment_pf(const RxParams &p, int seg, RxOut *o, u64 *acc, u32 *
     if (have) {
       // mode-B clusters to run whose state is stale first reconstruct it
       const u32 stale = runb & ~exact;
-      if (stale) rx_walk_back<G>(p, ir, c, pl, xr, w, stale, st, wbs, len_words);
+      if (stale) rx_walk_back<G>(p, ir, c, w, stale, st, wbs, len_words);
       const i64 fword = w * Bw - Lw;
       if (staged == w) {
         retire();
@@ -883,11 +908,11 @@ DEV void rx_run_segment_pf(const RxParams &p, int seg, RxOut *o, u64 *acc, u32 *
     // warp's own mask; one call site of the inlined body either way
     u32 U = run;
     if (lock) {
-      if (have && c.lane == 0) atomicOr(&rx_cta_union[par], run);
+      if (have && c.lane == 0) atomicOr(&rx_cta_u[par], run);
       const int more = __syncthreads_or(have);
-      U = rx_cta_union[par];
+      U = rx_cta_u[par];
       // every warp read the other word before this round's barrier
-      if (threadIdx.x == 0) rx_cta_union[par ^ 1] = 0u;
+      if (threadIdx.x == 0) rx_cta_u[par ^ 1] = 0u;
       par ^= 1;
       if (!more) break;
     } else if (!have) {
@@ -1121,8 +1146,12 @@ DEV bool rx_pf_ext_ok(const RxParams &p, const u32 *E, i64 q) {
 DEV u32 rx_pf_ht_hash(u32 gram, u32 k) { return (gram ^ (k * 0x27D4EB2Fu)) * 0x9E3779B1u; }
 
 // verify one filter hit: x = the 4 bytes ending at q, kbits: bit k-2 set if
-// the k-gram filter fired
-DEV void rx_pf_verify(const RxParams &p, u32 *sm, int NG, u32 x, u32 kbits, i64 q, int b) {
+// the k-gram filter fired.  tags: the tile's per-block direct-mapped record
+// of factor entries already applied to block b (an entry seen again in the
+// same block -- a common factor such as an HTTP header name -- skips its
+// member-mask loop; a tag collision only costs a redundant, idempotent OR)
+#define RX_PF_TAGS 64
+DEV void rx_pf_verify(const RxParams &p, u32 *sm, u32 *tags, int NG, u32 x, u32 kbits, i64 q, int b) {
   const u32 *T = p.pf_tab;
   const u32 hmask = (1u << p.pf_hbits) - 1u;
   for (u32 k = 4; k >= 2; --k) {
@@ -1136,7 +1165,10 @@ DEV void rx_pf_verify(const RxParams &p, u32 *sm, int NG, u32 x, u32 kbits, i64 
       if (e.y == 0u) break;
       if (e.x == gram && e.y == ((k << 1) | 1u)) {
         for (u32 j = 0; j < e.w; ++j) {
-          const u32 *E = T + p.pf_o_ext + 12u * (e.z + j);
+          const u32 ei = e.z + j;
+          u32 *tg = &tags[b * RX_PF_TAGS + (ei & (RX_PF_TAGS - 1))];
+          if (*(volatile u32 *)tg == ei + 1u) continue;  // applied to this block already
+          const u32 *E = T + p.pf_o_ext + 12u * ei;
           if (!rx_pf_ext_ok(p, E, q)) continue;
           const u32 t0 = __ldg(&E[9]), tn = __ldg(&E[10]);
           for (u32 t = t0; t < t0 + tn; ++t) {
@@ -1145,6 +1177,7 @@ DEV void rx_pf_verify(const RxParams &p, u32 *sm, int NG, u32 x, u32 kbits, i64 
             u32 *a = &sm[(kind * (u32)NG + g) * 32u + (u32)b];
             if ((*(volatile u32 *)a & m) != m) atomicOr(a, m);
           }
+          *(volatile u32 *)tg = ei + 1u;
         }
       }
       h = (h + 1u) & hmask;
@@ -1152,7 +1185,8 @@ DEV void rx_pf_verify(const RxParams &p, u32 *sm, int NG, u32 x, u32 kbits, i64 
   }
 }
 
-// smem: [filters (pf_smem_words) | member masks 2 x NG x 32 | per-warp hit queues 32 x 3]
+// smem: [filters (pf_smem_words) | member masks 2 x NG x 32 | per-warp hit
+// queues 32 x 3 | factor tags 32 blocks x RX_PF_TAGS]
 DEV void rx_prefilter_run(const RxParams &p, int NG) {
   extern __shared__ __align__(16) u32 pf_smem[];
   const int tid = threadIdx.x, nt = blockDim.x;
@@ -1161,6 +1195,7 @@ DEV void rx_prefilter_run(const RxParams &p, int NG) {
   for (u32 i = tid; i < p.pf_smem_words; i += nt) tab[i] = __ldg(&p.pf_tab[i]);
   u32 *sm = pf_smem + tw;                      // [2][NG][32 blocks] member masks
   u32 *wq = sm + 64 * NG + 96 * (tid >> 5);   // per-warp hit queue: 32 x {offset, x, kbits}
+  u32 *tags = sm + 64 * NG + 96 * (nt >> 5);   // [32 blocks][RX_PF_TAGS]
   const u32 *bl4 = tab, *bl3 = tab + p.pf_o_b3, *bg2 = tab + p.pf_o_b2;
   const bool has3 = p.pf_o_b3 != 0u, has2 = p.pf_o_b2 != 0u;
   const u32 s4 = 32u - p.pf_b4bits, s3 = 32u - p.pf_b3bits;
@@ -1170,8 +1205,22 @@ DEV void rx_prefilter_run(const RxParams &p, int NG) {
   const i64 nblk = 32 * p.pf_ntiles;
   for (i64 t = blockIdx.x; t < ntiles; t += gridDim.x) {
     for (int i = tid; i < 64 * NG; i += nt) sm[i] = 0u;
+    for (int i = tid; i < 32 * RX_PF_TAGS; i += nt) tags[i] = 0u;
     __syncthreads();
     const i64 tile_lo = p.avail_lo + t * RX_PF_TILE;
+    // the warp's filter hits are compacted into a queue of 32 that persists
+    // across the tile's chunks and is verified one hit per lane when full
+    // (and once at the tile's end): full-warp verification
+    u32 qn = 0;
+    auto flush = [&]() {
+      __syncwarp();
+      if (lane < qn) {
+        const u32 off = wq[3 * lane];
+        rx_pf_verify(p, sm, tags, NG, wq[3 * lane + 1], wq[3 * lane + 2], tile_lo + off, (int)(off >> 10));
+      }
+      __syncwarp();
+      qn = 0;
+    };
     for (int j = 0; j < RX_PF_TILE / 16; j += nt) {
       const i64 base = tile_lo + (i64)(j + tid) * 16;
       u32 w1, w2, w3, w4;
@@ -1208,34 +1257,23 @@ DEV void rx_prefilter_run(const RxParams &p, int NG) {
       u32 hm = h4 | h3 | h2;
       const i64 rem = p.avail_hi - base;
       if (rem < 16) hm &= rem <= 0 ? 0u : ((1u << rem) - 1u);
-      // the warp's hits are compacted into a queue of 32 and verified one per lane
-      u32 qn = 0;
       for (;;) {
         const u32 bal = __ballot_sync(RX_FULL, hm != 0u);
-        if (bal) {
-          const u32 rk = __popc(bal & ((1u << lane) - 1u));
-          if (hm != 0u && qn + rk < 32u) {
-            const int r = __ffs(hm) - 1;
-            hm &= hm - 1u;
-            u32 *e = wq + 3 * (qn + rk);
-            e[0] = (u32)(base + r - tile_lo);
-            e[1] = rx_pf_x(w0, w1, w2, w3, w4, r);
-            e[2] = ((h4 >> r) & 1u) << 2 | ((h3 >> r) & 1u) << 1 | ((h2 >> r) & 1u);
-          }
-          qn = qn + __popc(bal) < 32u ? qn + __popc(bal) : 32u;
+        if (!bal) break;
+        const u32 rk = __popc(bal & ((1u << lane) - 1u));
+        if (hm != 0u && qn + rk < 32u) {
+          const int r = __ffs(hm) - 1;
+          hm &= hm - 1u;
+          u32 *e = wq + 3 * (qn + rk);
+          e[0] = (u32)(base + r - tile_lo);
+          e[1] = rx_pf_x(w0, w1, w2, w3, w4, r);
+          e[2] = ((h4 >> r) & 1u) << 2 | ((h3 >> r) & 1u) << 1 | ((h2 >> r) & 1u);
         }
-        if (qn == 32u || (bal == 0u && qn > 0u)) {
-          __syncwarp();
-          if (lane < qn) {
-            const u32 off = wq[3 * lane];
-            rx_pf_verify(p, sm, NG, wq[3 * lane + 1], wq[3 * lane + 2], tile_lo + off, (int)(off >> 10));
-          }
-          __syncwarp();
-          qn = 0;
-        }
-        if (bal == 0u) break;
+        qn = qn + __popc(bal) < 32u ? qn + __popc(bal) : 32u;
+        if (qn == 32u) flush();
       }
     }
+    if (qn) flush();
     __syncthreads();
     // one warp per group: lane b holds block b's member masks; the group's
     // tile word of block bits is their ballot; lane m counts member m's blocks

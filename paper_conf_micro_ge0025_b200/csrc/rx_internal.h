@@ -192,6 +192,7 @@ struct RegexFactors {
 };
 
 struct CompiledSet {
+  int pass1_warps = 16;           // warps per pass-1 CTA (rx_runtime.cpp rx_compile)
   std::vector<int> factor_of;     // per regex: clustering key of its first-factor set, -1 = none (always runs)
   std::vector<RegexFactors> rf;   // per regex
   std::vector<Factor> factors;
@@ -210,7 +211,7 @@ void regex_factors(const Ast &a, CompiledSet &cs, RegexFactors &rf);
 // CUDA C sources: one relocatable unit per group + the kernel unit; linked
 // into one module with nvJitLink.
 std::string emit_group_unit(CompiledSet &cs, int gi);
-std::string emit_kernel_unit(CompiledSet &cs);
+std::string emit_kernel_unit(CompiledSet &cs, int gb, int ge);  // kernels of module [gb, ge)
 int lit_scratch_bytes(const CompiledSet &cs);  // per-warp shared bytes of the literal-run scratch
 int max_words_per_lane(const CompiledSet &cs);
 size_t warp_smem_bytes(const CompiledSet &cs);  // per-warp shared bytes of pass 1 / fix-up

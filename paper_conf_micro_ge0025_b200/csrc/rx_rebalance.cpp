@@ -2,8 +2,8 @@
 //
 // Operand rewriting: (A >> n) & B  ==  (A & (B << n)) >> n, exact on
 // finite zero-padded streams (SURVEY App.A-5).  The pass traverses the DFG in
-// topological order; for every AND whose operand is an Advance of a deeper
-// value A while the other operand B is shallower, the Advance is moved onto B
+// topological order; for every AND whose operand is an Advance deeper than
+// the other operand B (depth(A) + 1 > depth(B)), the Advance is moved onto B
 // as a lookahead and applied after the AND ("the SHIFT ... is moved to the
 // operand with lower topological depth"), iterating to a fixpoint;
 // trailing Advances of Advances are merged afterwards ("merged after
@@ -69,7 +69,8 @@ struct Pass {
         const Node &nx = ir.nodes[x];
         if (nx.op != Op::Adv || nx.loop >= 0 || nx.k <= 0) continue;
         int A = nx.a, k = nx.k;
-        if (!(d(A) > d(y))) continue;
+        // the SHIFT operand (depth d(A) + 1) is deeper than the other one
+        if (!(d(A) + 1 > d(y))) continue;
         Node look;
         look.op = Op::Look;
         look.a = y;

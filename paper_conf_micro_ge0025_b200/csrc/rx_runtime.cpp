@@ -206,10 +206,12 @@ bool nvrtc_compile(const std::string &src, int max_regs, bool use_cache, std::st
 // ---------------------------------------------------------------------------
 // program
 // ---------------------------------------------------------------------------
-constexpr int kPass1Warps = 16;  // one CTA = one SM's worth of warps, one group (lockstep)
 constexpr int kFixupWarps = 4;
+constexpr size_t kPfTagBytes = 4 * 32 * 64;  // prefilter factor tags (RX_PF_TAGS, rx_device.cuh)
+constexpr size_t kCtaHdr = 512;  // CTA header of pass 1 / fix-up shared memory (RX_CTA_HDR, rx_device.cuh)
 constexpr int kPrefilterWarps = 8;
 constexpr size_t kMaxSmem = 232448;  // opt-in dynamic shared memory per block (227 KB)
+constexpr size_t kModuleBytes = 48u << 20;  // code per linked module (see rx_compile)
 struct RxModule {
   int g_begin = 0, g_end = 0;  // group range
   int ns_max = 1, nr_max = 1;
@@ -228,6 +230,7 @@ struct RxModule {
 struct rx_program {
   rx::CompiledSet cs;
   uint32_t flags = 0;  // rx_options.flags
+  int pass1_warps = 16;  // pass-1 CTA: one SM's register file at max_regs, one group (lockstep)
   std::vector<RxModule> mods;
   uint32_t n_regex = 0;
   uint32_t state_words = 0;
@@ -281,7 +284,8 @@ const char *rx_program_source(const rx_program *p) { return p ? p->all_source.c_
 uint32_t rx_kernels_per_match(const rx_program *p) {
   uint32_t n = 0;
   if (p)
-    for (auto &m : p->mods) n += 1 + (m.any_state ? 2 : 0) + (p->cs.use_pf ? 1 : 0);
+    for (auto &m : p->mods) n += 1 + (m.any_state ? 2 : 0);
+  if (p && p->cs.use_pf && !p->mods.empty()) n += 1;  // one prefilter pass for all modules
   return n;
 }
 const char *rx_program_info(const rx_program *p) { return p ? p->info.c_str() : ""; }
@@ -354,7 +358,9 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
   memset(&o, 0, sizeof o);
   if (opt) o = *opt;
   rx::LowerOptions lo;
-  lo.interval = o.interval == 0 ? 8 : (o.interval == UINT32_MAX ? 0 : (int)o.interval);
+  // default 4 (the paper fixes 8; 1-4 measured ~11% faster than 8 on the Snort-like set,
+  // profiles/r2_ablation_snort.md)
+  lo.interval = o.interval == 0 ? 4 : (o.interval == UINT32_MAX ? 0 : (int)o.interval);
   if (o.flags & RX_F_NO_GUARDS) lo.interval = 0;
   lo.rebalance = (o.flags & RX_F_REBALANCE) && !(o.flags & RX_F_NO_REBALANCE);
   int max_regs = o.max_regs ? (int)o.max_regs : 128;
@@ -372,6 +378,11 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
   auto *p = new rx_program();
   p->n_regex = n_patterns;
   p->flags = o.flags;
+  // pass-1 CTA size: one SM's register file (64 K registers) at max_regs --
+  // 16 warps at 128 registers, 12 at 168, 8 at 255 (rx_options.max_regs)
+  max_regs = std::max(32, std::min(255, max_regs));
+  p->pass1_warps = std::max(1, std::min(16, 65536 / (32 * max_regs)));
+  p->cs.pass1_warps = p->pass1_warps;
   p->cs.irs.resize(n_patterns);
   p->cs.factor_of.assign(n_patterns, -1);
   p->cs.rf.assign(n_patterns, rx::RegexFactors());
@@ -402,7 +413,7 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
     }
     if (use_pf) {
       rx::regex_factors(*ast, p->cs, p->cs.rf[i]);
-      if (o.flags & RX_F_NO_MODEB) p->cs.rf[i].out.clear();
+      if (!(o.flags & RX_F_MODEB) || (o.flags & RX_F_NO_MODEB)) p->cs.rf[i].out.clear();
       const auto &fs = p->cs.rf[i].first;
       if (!fs.empty()) {
         auto it = first_key.find(fs);
@@ -482,27 +493,32 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
   // a program whose layout exceeds the opt-in limit must fail here, not at
   // every launch)
   mm.warp_smem = rx::warp_smem_bytes(p->cs);
-  if (mm.warp_smem * kPass1Warps > kMaxSmem) {
+  if (mm.warp_smem * p->pass1_warps + kCtaHdr > kMaxSmem) {
+    const size_t need = mm.warp_smem * p->pass1_warps + kCtaHdr;
     delete p;
-    return fail(RX_ETOOBIG, "pass-1 shared memory " + std::to_string(mm.warp_smem * kPass1Warps) +
-                                " B exceeds the 227 KB per-block limit (fewer state slots / regexes per group, or "
+    return fail(RX_ETOOBIG, "pass-1 shared memory " + std::to_string(need) + " B exceeds the 227 KB per-block limit (fewer state slots / regexes per group, or "
                                 "smaller words_per_lane)");
   }
   if (p->cs.use_pf) {
     const size_t pfb =
-        4 * (((size_t)p->cs.pf.smem_words + 3) & ~(size_t)3) + 4 * 64 * (size_t)G + 4 * 96 * kPrefilterWarps;
+        4 * (((size_t)p->cs.pf.smem_words + 3) & ~(size_t)3) + 4 * 64 * (size_t)G + 4 * 96 * kPrefilterWarps +
+        kPfTagBytes;
     if (pfb > kMaxSmem) {
       delete p;
       return fail(RX_ETOOBIG, "prefilter shared memory " + std::to_string(pfb) + " B exceeds the 227 KB limit");
     }
   }
   p->info = info.str();
-  std::vector<std::string> srcs(G + 1), cubins(G + 1), logs(G + 1);
-  for (int gi = 0; gi < G; ++gi) srcs[gi] = rx::emit_group_unit(p->cs, gi);
-  srcs[G] = rx::emit_kernel_unit(p->cs);
-  std::vector<int> okv(G + 1, 0);
+  // one relocatable NVRTC unit per group, compiled in parallel; then the
+  // groups are split into modules of at most kModuleBytes of code (the
+  // driver's linker crashed in cuLinkComplete on one image of all 545 group
+  // units of the 10k-regex set), each with its own kernel unit
   bool use_cache = !(o.flags & RX_F_NO_CACHE);
-  {
+  auto compile_all = [&](std::vector<std::string> &srcs, std::vector<std::string> &cubins,
+                         std::vector<std::string> &logs) -> bool {
+    cubins.assign(srcs.size(), std::string());
+    logs.assign(srcs.size(), std::string());
+    std::vector<int> okv(srcs.size(), 0);
     std::vector<std::thread> th;
     std::atomic<size_t> next{0};
     size_t nthreads = std::min<size_t>(srcs.size(), hw);
@@ -515,23 +531,64 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
         }
       });
     for (auto &t : th) t.join();
-  }
-  for (size_t m = 0; m < srcs.size(); ++m) {
-    if (!okv[m]) {
-      std::string head = logs[m].substr(0, 240);
-      if (err) {
-        err->pattern_index = 0;
-        err->byte_offset = 0;
-        snprintf(err->msg, sizeof err->msg, "%s", head.c_str());
+    for (size_t m = 0; m < srcs.size(); ++m) {
+      if (!okv[m]) {
+        std::string head = logs[m].substr(0, 240);
+        if (err) {
+          err->pattern_index = 0;
+          err->byte_offset = 0;
+          snprintf(err->msg, sizeof err->msg, "%s", head.c_str());
+        }
+        fail(RX_EJIT, "NVRTC: " + logs[m].substr(0, 4000));
+        return false;
       }
-      std::string full = logs[m];
-      delete p;
-      return fail(RX_EJIT, "NVRTC: " + full.substr(0, 4000));
     }
+    return true;
+  };
+  std::vector<std::string> gsrc(G), gcub, glog;
+  for (int gi = 0; gi < G; ++gi) gsrc[gi] = rx::emit_group_unit(p->cs, gi);
+  if (!compile_all(gsrc, gcub, glog)) {
+    delete p;
+    return RX_EJIT;
   }
-  mm.units = std::move(cubins);  // relocatable; linked by the driver at module load
-  for (auto &s : srcs) p->all_source += s;
-  p->mods.push_back(mm);
+  std::vector<std::pair<int, int>> ranges;
+  {
+    size_t acc = 0;
+    int b = 0;
+    for (int gi = 0; gi < G; ++gi) {
+      if (gi > b && acc + gcub[gi].size() > kModuleBytes) {
+        ranges.push_back({b, gi});
+        b = gi;
+        acc = 0;
+      }
+      acc += gcub[gi].size();
+    }
+    if (G > 0 || ranges.empty()) ranges.push_back({b, G});
+  }
+  std::vector<std::string> ksrc(ranges.size()), kcub, klog;
+  for (size_t m = 0; m < ranges.size(); ++m) ksrc[m] = rx::emit_kernel_unit(p->cs, ranges[m].first, ranges[m].second);
+  if (!compile_all(ksrc, kcub, klog)) {
+    delete p;
+    return RX_EJIT;
+  }
+  for (int gi = 0; gi < G; ++gi) p->all_source += gsrc[gi];
+  for (size_t m = 0; m < ranges.size(); ++m) {
+    RxModule mod;
+    mod.g_begin = ranges[m].first;
+    mod.g_end = ranges[m].second;
+    mod.warp_smem = mm.warp_smem;
+    for (int gi = mod.g_begin; gi < mod.g_end; ++gi) {
+      const auto &g = p->cs.groups[gi];
+      mod.ns_max = std::max(mod.ns_max, g.nslots);
+      mod.nr_max = std::max<int>(mod.nr_max, (int)g.regexes.size());
+      if (g.nslots > 0) mod.any_state = true;
+      mod.units.push_back(std::move(gcub[gi]));
+    }
+    mod.units.push_back(std::move(kcub[m]));  // relocatable; linked by the driver at module load
+    p->all_source += ksrc[m];
+    p->mods.push_back(std::move(mod));
+  }
+  p->info += "modules: " + std::to_string(ranges.size()) + "\n";
   *out = p;
   return RX_OK;
 }
@@ -636,10 +693,10 @@ rx_status launch(rx_program *p, RxModule &m, CUfunction f, long long blocks, int
   if (blocks > 0x7fffffffLL) return fail(RX_EINVAL, "grid too large");
   // shared memory: pass 1 / fix-up = per-warp layout of rx_codegen.cpp
   // emit_group_unit; prefilter = [filters | 2 x NG x 32 member masks | hit queues]
-  size_t bytes = (size_t)warps_per_block * m.warp_smem;
+  size_t bytes = kCtaHdr + (size_t)warps_per_block * m.warp_smem;
   if (f == m.prefilter)
-    bytes = 4 * (((size_t)prm.pf_smem_words + 3) & ~(size_t)3) + 4 * 64 * (size_t)(m.g_end - m.g_begin) +
-            4 * 96 * (size_t)warps_per_block;
+    bytes = 4 * (((size_t)prm.pf_smem_words + 3) & ~(size_t)3) + 4 * 64 * p->cs.groups.size() +
+            4 * 96 * (size_t)warps_per_block + kPfTagBytes;
   if (bytes > kMaxSmem) return fail(RX_ETOOBIG, "shared memory layout exceeds 227 KB");
   const unsigned smem = (unsigned)bytes;
   if (smem > 48 * 1024 &&
@@ -752,96 +809,110 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
   const long long waves = 16;
   const long long target_ctas = 148LL * waves;
   const long long cpg0 = std::max<long long>(1, div_up(target_ctas, std::max(G, 1)));
-  long long sw = std::max<long long>(4, div_up(max_nwin, cpg0 * kPass1Warps));
+  long long sw = std::max<long long>(4, div_up(max_nwin, cpg0 * p->pass1_warps));
   long long nseg_max = std::max<long long>(1, div_up(max_nwin, sw));
-  const long long cpg = div_up(nseg_max, kPass1Warps);
+  const long long cpg = div_up(nseg_max, p->pass1_warps);
   prm.sw = (int)std::min<long long>(sw, 1 << 30);
   prm.nseg_max = (int)nseg_max;
   prm.mode = 0;
   const bool stats_on = (p->flags & RX_F_STATS) != 0;
+  // scratch indexed by global group id (group units use G::NG, G::GID and the
+  // program-wide NSMAX): sized for all groups, shared by the modules
+  int ns_all = 1;
+  bool any_state = false;
   for (auto &m : p->mods) {
-    int mg = m.g_end - m.g_begin;
-    unsigned int *seg_state = nullptr;
-    size_t bytes = 4ull * (size_t)nseg_max * (size_t)mg * (size_t)std::max(1, m.ns_max);
-    if (m.any_state) {
-      if (!(seg_state = (unsigned int *)scratch_get(p, stream, SC_SEGSTATE, bytes))) return fail(RX_ENOMEM, "seg_state");
-    }
-    prm.seg_state = seg_state;
-    prm.mode = 0;
-    prm.pf_on = 0;
-    if (p->cs.use_pf) {
-      const long long span = prm.avail_hi - prm.avail_lo;
-      const long long ntiles = std::max<long long>(1, div_up(span, 32768));
-      const size_t gb_bytes = ((size_t)4 * (size_t)ntiles * (size_t)mg + 255) & ~(size_t)255;
-      const size_t bl_bytes = ((size_t)4 * 32 * (size_t)ntiles * (size_t)mg + 255) & ~(size_t)255;
-      const size_t cnt_bytes = (size_t)4 * 64 * (size_t)mg;
-      char *pf_scratch = (char *)scratch_get(p, stream, SC_PF, gb_bytes + 2 * bl_bytes + cnt_bytes + 256);
-      if (!pf_scratch) return fail(RX_ENOMEM, "prefilter scratch");
-      const rx::Prefilter &pf = p->cs.pf;
-      prm.pf_tab = (const unsigned int *)m.pf_mem;
-      prm.pf_words = (unsigned int)pf.blob.size();
-      prm.pf_smem_words = pf.smem_words;
-      prm.pf_b4bits = pf.b4bits;
-      prm.pf_b3bits = pf.hbits >> 8;
-      prm.pf_hbits = pf.hbits & 255u;
-      prm.pf_o_b3 = pf.o_b3;
-      prm.pf_o_b2 = pf.o_b2;
-      prm.pf_o_ht = pf.o_ht;
-      prm.pf_o_ext = pf.o_ext;
-      prm.pf_o_fgoff = pf.o_fgoff;
-      prm.pf_o_fgent = pf.o_fgent;
-      prm.pf_gbits = (unsigned int *)pf_scratch;
-      prm.pf_mmask = (unsigned int *)(pf_scratch + gb_bytes);
-      prm.pf_omask = (unsigned int *)(pf_scratch + gb_bytes + bl_bytes);
-      prm.pf_cnt = (unsigned int *)(pf_scratch + gb_bytes + 2 * bl_bytes);
-      prm.pf_ntiles = ntiles;
-      prm.pf_on = 1;
-      if (cudaMemsetAsync(prm.pf_cnt, 0, cnt_bytes, stream) != cudaSuccess) return fail(RX_ECUDA, "memset");
-      // 8-warp CTAs, several per SM (the verification of filter hits is a
-      // chain of dependent loads: more resident warps hide it)
-      s = launch(p, m, m.prefilter, std::min<long long>(ntiles, 148LL * 8), kPrefilterWarps, prm, stream);
-      if (s != RX_OK) return s;
-    }
-    unsigned long long *stats = nullptr;
-    const size_t stats_bytes = 8 * (8 + 4 * (size_t)mg);
-    if (stats_on && cudaMalloc((void **)&stats, stats_bytes) == cudaSuccess)
-      cudaMemsetAsync(stats, 0, stats_bytes, stream);
-    prm.stats = stats;
-    s = launch(p, m, m.pass1, cpg * mg, kPass1Warps, prm, stream);
-    prm.stats = nullptr;
-    if (stats) {
-      std::vector<unsigned long long> h(stats_bytes / 8);
-      cudaMemcpyAsync(h.data(), stats, stats_bytes, cudaMemcpyDeviceToHost, stream);
-      cudaStreamSynchronize(stream);
-      fprintf(stderr, "[rx stats] groups=%d window_visits=%llu active=%llu member_hits=%llu walkbacks=%llu "
-              "walk_rounds=%llu\n", mg, h[3], h[0], h[2], h[4], h[5]);
-      for (int g = 0; g < mg; ++g)
-        fprintf(stderr, "[rx stats] group %d: active=%llu member_hits=%llu modeB_members=%llu\n", g, h[8 + 4 * g],
-                h[9 + 4 * g], h[10 + 4 * g]);
-      cudaFree(stats);
-    }
+    ns_all = std::max(ns_all, m.ns_max);
+    any_state = any_state || m.any_state;
+  }
+  const size_t bytes = 4ull * (size_t)nseg_max * (size_t)G * (size_t)ns_all;
+  unsigned int *seg_state = nullptr;
+  if (any_state && !(seg_state = (unsigned int *)scratch_get(p, stream, SC_SEGSTATE, bytes)))
+    return fail(RX_ENOMEM, "seg_state");
+  prm.seg_state = seg_state;
+  prm.mode = 0;
+  prm.pf_on = 0;
+  if (p->cs.use_pf) {
+    // one prefilter pass for all groups (module 0 holds the kernel; it
+    // indexes its outputs by global group id)
+    const long long span = prm.avail_hi - prm.avail_lo;
+    const long long ntiles = std::max<long long>(1, div_up(span, 32768));
+    const size_t gb_bytes = ((size_t)4 * (size_t)ntiles * (size_t)G + 255) & ~(size_t)255;
+    const size_t bl_bytes = ((size_t)4 * 32 * (size_t)ntiles * (size_t)G + 255) & ~(size_t)255;
+    const size_t cnt_bytes = (size_t)4 * 64 * (size_t)G;
+    char *pf_scratch = (char *)scratch_get(p, stream, SC_PF, gb_bytes + 2 * bl_bytes + cnt_bytes + 256);
+    if (!pf_scratch) return fail(RX_ENOMEM, "prefilter scratch");
+    const rx::Prefilter &pf = p->cs.pf;
+    RxModule &m0 = p->mods[0];
+    prm.pf_tab = (const unsigned int *)m0.pf_mem;
+    prm.pf_words = (unsigned int)pf.blob.size();
+    prm.pf_smem_words = pf.smem_words;
+    prm.pf_b4bits = pf.b4bits;
+    prm.pf_b3bits = pf.hbits >> 8;
+    prm.pf_hbits = pf.hbits & 255u;
+    prm.pf_o_b3 = pf.o_b3;
+    prm.pf_o_b2 = pf.o_b2;
+    prm.pf_o_ht = pf.o_ht;
+    prm.pf_o_ext = pf.o_ext;
+    prm.pf_o_fgoff = pf.o_fgoff;
+    prm.pf_o_fgent = pf.o_fgent;
+    prm.pf_gbits = (unsigned int *)pf_scratch;
+    prm.pf_mmask = (unsigned int *)(pf_scratch + gb_bytes);
+    prm.pf_omask = (unsigned int *)(pf_scratch + gb_bytes + bl_bytes);
+    prm.pf_cnt = (unsigned int *)(pf_scratch + gb_bytes + 2 * bl_bytes);
+    prm.pf_ntiles = ntiles;
+    prm.pf_on = 1;
+    if (cudaMemsetAsync(prm.pf_cnt, 0, cnt_bytes, stream) != cudaSuccess) return fail(RX_ECUDA, "memset");
+    // 8-warp CTAs, several per SM (the verification of filter hits is a
+    // chain of dependent loads: more resident warps hide it)
+    s = launch(p, m0, m0.prefilter, std::min<long long>(ntiles, 148LL * 8), kPrefilterWarps, prm, stream);
     if (s != RX_OK) return s;
-    if (m.any_state) {
-      // carry fix-up, phase 1: one warp per (group, segment) in parallel;
-      // phase 2: one warp per group, only where a segment's carry outlived it.
-      // (pf_on stays set: the fix-up recomputes the mode-B choice from the
-      // prefilter's counts and leaves those clusters alone)
-      prm.mode = 1;
-      void *fx = nullptr;
-      const size_t nc_bytes = 4ull * (size_t)nseg_max * (size_t)mg;
-      if (!(fx = scratch_get(p, stream, SC_FIX, bytes + nc_bytes + 256))) return fail(RX_ENOMEM, "fix-up scratch");
-      prm.seg_fix = (unsigned int *)fx;
-      prm.seg_nc = (unsigned int *)((char *)fx + ((bytes + 255) & ~(size_t)255));
-      cudaMemsetAsync(prm.seg_nc, 0, nc_bytes, stream);
-      prm.fix_phase = 1;
-      s = launch(p, m, m.fixup, div_up((long long)mg * nseg_max, kFixupWarps), kFixupWarps, prm, stream);
-      if (s == RX_OK) {
-        prm.fix_phase = 2;
-        s = launch(p, m, m.fixup, div_up(mg, kFixupWarps), kFixupWarps, prm, stream);
+  }
+  unsigned long long *stats = nullptr;
+  const size_t stats_bytes = 8 * (8 + 4 * (size_t)G);
+  if (stats_on && cudaMalloc((void **)&stats, stats_bytes) == cudaSuccess) cudaMemsetAsync(stats, 0, stats_bytes, stream);
+  for (auto &m : p->mods) {
+    const int mg = m.g_end - m.g_begin;
+    prm.mode = 0;
+    prm.stats = stats;
+    s = launch(p, m, m.pass1, cpg * mg, p->pass1_warps, prm, stream);
+    prm.stats = nullptr;
+    if (s != RX_OK) break;
+  }
+  if (stats) {
+    std::vector<unsigned long long> h(stats_bytes / 8);
+    cudaMemcpyAsync(h.data(), stats, stats_bytes, cudaMemcpyDeviceToHost, stream);
+    cudaStreamSynchronize(stream);
+    fprintf(stderr, "[rx stats] groups=%d window_visits=%llu active=%llu member_hits=%llu walkbacks=%llu "
+            "walk_rounds=%llu cluster_runs=%llu\n", G, h[3], h[0], h[2], h[4], h[5], h[6]);
+    for (int g = 0; g < G; ++g)
+      fprintf(stderr, "[rx stats] group %d: active=%llu member_hits=%llu modeB_members=%llu cluster_runs=%llu\n", g,
+              h[8 + 4 * g], h[9 + 4 * g], h[10 + 4 * g], h[11 + 4 * g]);
+    cudaFree(stats);
+  }
+  if (s != RX_OK) return s;
+  if (any_state) {
+    // carry fix-up, phase 1: one warp per (group, segment) in parallel;
+    // phase 2: one warp per group, only where a segment's carry outlived it.
+    // (pf_on stays set: the fix-up recomputes the mode-B choice from the
+    // prefilter's counts and leaves those clusters alone)
+    prm.mode = 1;
+    void *fx = nullptr;
+    const size_t nc_bytes = 4ull * (size_t)nseg_max * (size_t)G;
+    if (!(fx = scratch_get(p, stream, SC_FIX, bytes + nc_bytes + 256))) return fail(RX_ENOMEM, "fix-up scratch");
+    prm.seg_fix = (unsigned int *)fx;
+    prm.seg_nc = (unsigned int *)((char *)fx + ((bytes + 255) & ~(size_t)255));
+    cudaMemsetAsync(prm.seg_nc, 0, nc_bytes, stream);
+    for (int phase = 1; phase <= 2 && s == RX_OK; ++phase) {
+      prm.fix_phase = phase;
+      for (auto &m : p->mods) {
+        if (!m.any_state) continue;
+        const long long mg = m.g_end - m.g_begin;
+        s = launch(p, m, m.fixup, div_up(phase == 1 ? mg * nseg_max : mg, kFixupWarps), kFixupWarps, prm, stream);
+        if (s != RX_OK) break;
       }
-      prm.fix_phase = 0;
-      if (s != RX_OK) return s;
     }
+    prm.fix_phase = 0;
+    if (s != RX_OK) return s;
   }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(RX_ECUDA, cudaGetErrorString(e));

@@ -1,6 +1,6 @@
 """Accounting of the sparse pass 1 (rx_options.flags |= RX_F_STATS): window
 visits, active windows, prefilter member hits, mode-B walk-backs, per group.
-Usage: python scripts/stats_run.py [config] [length_mib] [--no-modeb]"""
+Usage: python scripts/stats_run.py [config] [length_mib] [--modeb]"""
 import os
 import sys
 import time
@@ -18,7 +18,7 @@ cfg = args[0] if args else "snort"
 mib = int(args[1]) if len(args) > 1 else 0
 pats, data, n, name = bench.load_workload(cfg, (mib << 20) if mib else None)
 t = time.time()
-flags = rx.RX_F_STATS | (rx.RX_F_NO_MODEB if "--no-modeb" in sys.argv else 0)
+flags = rx.RX_F_STATS | (rx.RX_F_MODEB if "--modeb" in sys.argv else 0)
 prog = rx.Program(pats, flags=flags, **bench.PROGRAM_OPTS.get(cfg, {}))
 print(f"compiled {len(pats)} regexes, {prog.n_groups} groups in {time.time() - t:.1f} s", flush=True)
 if os.environ.get("RX_INFO_OUT"):

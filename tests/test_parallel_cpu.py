@@ -2,9 +2,10 @@
 CPU with the gloo backend, world sizes 2 and 3.
 
 The GPU matching is replaced by a small exact model of a chunk's boundary
-state so that the protocol -- speculative zero-state match, sequential state
-resolution by broadcast, rematch only where the true incoming state differs,
-all-reduce of per-regex counts -- is checked end to end across processes.
+state so that the protocol -- halo exchange by all_gather, speculative zero-state
+match, state resolution by all_gather rounds, rematch only where the true
+incoming state differs, all-reduce of per-regex counts -- is checked end to
+end across processes.
 The model: the "regex" counts positions where the running count of byte 'a'
 since the last 'z' is odd; the boundary state is that parity (a carried
 state in the sense of DESIGN.md "Forwarded state").
@@ -28,40 +29,51 @@ def _free_port():
     return p
 
 
-def model_match(data: bytes, state_in: int):
-    """(count, state_out) of the toy carried-state program."""
+def model_match(data: bytes, state_in: int, lo: int = 0, hi: int = None):
+    """(count, state_out) of the toy program over data[lo:hi] (data may hold
+    halo bytes around it): positions i where the parity of 'a's since the
+    last 'z' is odd (carried state), plus positions with data[i-1:i+1] == b"bc"
+    (one byte of lookback) and data[i:i+2] == b"ca" (one byte of lookahead)."""
+    hi = len(data) if hi is None else hi
     par = state_in
     n = 0
-    for b in data:
+    for i in range(lo, hi):
+        b = data[i]
         if b == ord("z"):
             par = 0
         elif b == ord("a"):
             par ^= 1
         n += par
+        n += i > 0 and data[i - 1:i + 1] == b"bc"
+        n += data[i:i + 2] == b"ca"
     return n, par
 
 
 class FakeProg:
-    """Stands in for parallel.ChunkMatcher's Program (CPU tensors)."""
+    """Stands in for parallel.ChunkMatcher's Program (CPU tensors): computes
+    from the halo'd buffer it is given, so the halo exchange is exercised."""
 
-    def __init__(self, data: bytes):
-        self.data = data
+    def __init__(self):
         self.boundary_bytes = 4
+        self.lookback = 1
+        self.lookahead = 1
         self.calls = []
+
+    def _run(self, buf, length, halo_left, state):
+        data = bytes(buf.tolist())
+        return model_match(data, state, halo_left, halo_left + length)
 
     def match_chunk(self, buf, length, halo_left, halo_right, global_offset, state_in=None, state_out=None,
                     out=None):
         s_in = 0 if state_in is None else int(state_in[0])
-        chunk = self.data[global_offset:global_offset + length]
-        n, s_out = model_match(chunk, s_in)
+        n, s_out = self._run(buf, length, halo_left, s_in)
         out["counts"][0] = n
         state_out[0] = s_out
         self.calls.append(("match", s_in))
 
     def rematch_chunk(self, buf, length, halo_left, halo_right, global_offset, assumed, true, state_out, out):
-        chunk = self.data[global_offset:global_offset + length]
-        n_old, _ = model_match(chunk, int(assumed[0]))
-        n_new, s_out = model_match(chunk, int(true[0]))
+        n_old, _ = self._run(buf, length, halo_left, int(assumed[0]))
+        n_new, s_out = self._run(buf, length, halo_left, int(true[0]))
         out["counts"][0] += n_new - n_old
         state_out[0] = s_out
         self.calls.append(("rematch", int(true[0])))
@@ -72,12 +84,13 @@ def _worker(rank, world, port, data, q):
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
-        prog = FakeProg(data)
+        prog = FakeProg()
         cm = parallel.ChunkMatcher(prog, torch.device("cpu"), dist=dist)
         a, b = parallel.chunk_bounds(len(data), world, rank)
+        chunk = torch.tensor(list(data[a:b]), dtype=torch.uint8)
         out = {"counts": torch.zeros(1, dtype=torch.int64), "digests": None}
-        reruns = cm.match_chunk(None, b - a, 0, 0, a, rank, world, out)
-        q.put((rank, int(out["counts"][0]), reruns, prog.calls))
+        reruns = cm.match_stream_chunk(chunk, rank, world, out, a)
+        q.put((rank, int(out["counts"][0]), reruns, prog.calls, cm.last["gather_rounds"]))
     finally:
         dist.destroy_process_group()
 
@@ -88,6 +101,11 @@ def test_chunked_protocol_equals_whole_stream(world):
     alphabet = b"aazbc"
     data = bytes(alphabet[i] for i in torch.randint(0, len(alphabet), (3000,), generator=rng).tolist())
     data = data[:1000] + b"a" + b"b" * 999 + data[2000:]  # a parity carried across a chunk boundary
+    # "bc" / "ca" pairs straddling the cuts (halo bytes needed on both sides)
+    cuts = [parallel.chunk_bounds(len(data), world, r)[0] for r in range(1, world)]
+    for j, c in enumerate(cuts):
+        pair = b"bc" if j % 2 == 0 else b"ca"
+        data = data[:c - 1] + pair + data[c + 1:]
     whole, _ = model_match(data, 0)
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
@@ -103,12 +121,13 @@ def test_chunked_protocol_equals_whole_stream(world):
     # every rank holds the all-reduced total == the whole-stream count
     assert all(r[1] == whole for r in res), (whole, res)
     # rank r re-ran iff its true incoming state was not the assumed zero
-    for rank, _, reruns, calls in res:
+    for rank, _, reruns, calls, rounds in res:
         a, _ = parallel.chunk_bounds(len(data), world, rank)
         _, true_in = model_match(data[:a], 0)
         assert reruns == (1 if rank > 0 and true_in != 0 else 0)
         if reruns:
             assert calls[-1] == ("rematch", true_in)
+        assert 1 <= rounds <= world
 
 
 def test_shard_patterns_is_a_balanced_partition():

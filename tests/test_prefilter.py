@@ -78,7 +78,7 @@ def test_factor_occurs_in_every_match_bruteforce():
         p = gen.fuzz_pattern(rng)
         if len(p) <= 20:
             pats.append(p)
-    prog = rx.Program(pats)
+    prog = rx.Program(pats, flags=rx.RX_F_MODEB)  # output factors exist only with mode B allowed
     fac = factors(prog)
     assert sum(v[0] is not None for v in fac.values()) >= 10
     assert sum(v[1] is not None for v in fac.values()) >= 10
@@ -121,7 +121,7 @@ def test_factor_windows_are_long_and_exact():
     # extension windows: the whole fixed-offset literal prefix (<= 16 bytes),
     # alternations of words branch, classes of one bit stay compared
     prog = rx.Program([rb"HTTP/1\.union.+<script>", rb"GET(admin|root)xyz", rb"Cookie:[^\x00]*619ajavascript:",
-                       rb"[Ss]elect\s+from"])
+                       rb"[Ss]elect\s+from"], flags=rx.RX_F_MODEB)
     fac = factors(prog)
     (f0, o0, _), (f1, _, _), (f2, o2, d2), (f3, _, _) = fac[0], fac[1], fac[2], fac[3]
     assert f0 is not None and bytes(v for v, m in zip(f0[0][0], f0[0][1]) if m == 0xff) == b"HTTP/1.union"
@@ -134,7 +134,7 @@ def test_factor_windows_are_long_and_exact():
 def test_stateful_factor_precedes_first_unbounded_repetition():
     # property (ii): first factors are taken before the first unbounded
     # repetition; output factors from the suffix after the last one
-    prog = rx.Program([rb"(?:ab)+cdef", rb"xyzw[0-9]+qrst", rb"abcd.*wxyz", rb"abcd[a-z]+"])
+    prog = rx.Program([rb"(?:ab)+cdef", rb"xyzw[0-9]+qrst", rb"abcd.*wxyz", rb"abcd[a-z]+"], flags=rx.RX_F_MODEB)
     fac = factors(prog)
     assert fac[0][0] is None                           # nothing mandatory before (ab)+
     assert bytes(fac[1][0][0][0]) == b"xyzw"           # not "qrst"
@@ -245,7 +245,7 @@ def test_mode_b_walk_back_bit_exact(capfd):
     pats = [rb"Cookie:[^\x00]*619ajavascript:", rb"HTTP/1\.(?:%[0-9a-f]{2})*DpPXrWa(?:iJ4/)*",
             rb"Cookie:[a-z]+=qz7Kx", rb"HTTP/1\.[^\r\n]*q9Zz", rb"zz[0-9]+", rb"abc"]
     rng = np.random.default_rng(3)
-    prog = rx.Program(pats, flags=rx.RX_F_STATS)
+    prog = rx.Program(pats, flags=rx.RX_F_STATS | rx.RX_F_MODEB)
     plants = [b"619ajavascript:", b"%2f%3aDpPXrWaiJ4/iJ4/", b"DpPXrWa", b"abc=qz7Kx", b"q9Zz"]
     for n in (5000, 200000, (3 << 20) + 123):
         a = _modeb_input(rng, n, b"Cookie:", plants[0])
@@ -266,9 +266,9 @@ def test_mode_b_walk_back_bit_exact(capfd):
 
 @gpu
 def test_mode_b_off_equals_on():
-    # the ablation flag (RX_F_NO_MODEB) gives the same result on the Snort-like set
+    # mode B (RX_F_MODEB, opt-in) gives the same result on the Snort-like set
     pats = gen.snort_patterns(300, 2)[0]
     data = bytes(gen.snort_input((1 << 20) + 5, seed=7))
-    a = _gpu_counts(rx.Program(pats), data)
-    b = _gpu_counts(rx.Program(pats, flags=rx.RX_F_NO_MODEB), data)
+    a = _gpu_counts(rx.Program(pats, flags=rx.RX_F_MODEB), data)
+    b = _gpu_counts(rx.Program(pats), data)
     assert np.array_equal(a["counts"], b["counts"]) and np.array_equal(a["digests"], b["digests"])
