@@ -144,7 +144,47 @@ def ncu_traffic(workload: str, kernel: str, nbytes: int):
         return None
 
 
-def roofline(ktimes, nbytes, n_regex, hbm, hbm_src, workload, step_ms):
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return None
+
+
+def int_peak():
+    """Measured integer-pipe peak of this GPU (scripts/int_peak.cu, committed
+    as profiles/r2_int_peak.json): LOP3 / IADD3 / SHF / PRMT all issue at the
+    same rate -- the ALU pipe's -- which bounds the bitstream body."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "r2_int_peak.json")) as f:
+            d = json.load(f)
+        return float(d["rates"]["lop3"]["tops"]), "profiles/r2_int_peak.json (LOP3 rate, measured on a B200 at 1965 MHz)"
+    except Exception:
+        return None, None
+
+
+def int_block(workload, kernel, avg_ms, nbytes):
+    """Integer-pipe view of the dominant kernel: executed thread instructions
+    per launch (copied from the committed ncu capture named in `inst_source`,
+    scaled to this input) over its live duration, against the ALU peak."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+            e = json.load(f)[workload][kernel]
+        ti = float(e["thread_inst_per_launch"]) * nbytes / float(e["input_bytes"])
+    except Exception:
+        return None
+    peak, src = int_peak()
+    ach = ti / (avg_ms * 1e-3) / 1e12
+    return {"thread_ops_per_byte": ti / nbytes, "achieved": ach, "peak": peak, "unit": "Tops/s",
+            "frac": ach / peak if peak else None, "inst_source": "copied: " + str(e.get("source", "ncu")),
+            "peak_source": src}
+
+
+def roofline(ktimes, nbytes, n_regex, hbm, hbm_src, workload, step_ms, steps):
     """Roofline of the dominant kernel (the one with the largest share of the
     step): achieved = its ALGORITHMIC bytes per launch (the input, read once,
     plus 8 B of counts per regex -- DESIGN.md "Roofline") / its average launch
@@ -158,10 +198,14 @@ def roofline(ktimes, nbytes, n_regex, hbm, hbm_src, workload, step_ms):
     ach = alg / (avg_ms * 1e-3) / 1e9
     traffic = ncu_traffic(workload, k, nbytes)
     return {"bound": "hbm", "achieved": ach, "peak": hbm, "unit": "GB/s", "frac": ach / hbm,
-            "traffic": traffic, "kernel": k, "kernel_ms": avg_ms, "share_of_step": tot_ms / n / step_ms,
+            "traffic": traffic, "kernel": k, "kernel_ms": avg_ms, "share_of_step": tot_ms / steps / step_ms,
             "algorithmic_bytes_per_launch": alg, "peak_source": hbm_src,
-            "kernels_ms_per_step": {kk: vv[0] / max(vv[1], 1) for kk, vv in busy.items()},
-            "note": "the path is integer-ALU bound (DESIGN.md Roofline): %HBM is the metric's denominator"}
+            "kernels_ms_per_step": {kk: vv[0] / steps for kk, vv in busy.items()},
+            "launches_per_step": {kk: vv[1] / steps for kk, vv in busy.items()},
+            "traffic_source": "copied: profiles/ncu_traffic.json (ncu --set full dram__bytes_read+write per launch)",
+            "int": int_block(workload, k, avg_ms, nbytes),
+            "note": "%HBM is the metric's denominator; the kernels are bound by issue / latency of integer "
+                    "work (see int and DESIGN.md Roofline), not by DRAM"}
 
 
 def load_workload(config: str, length=None, rank: int = 0):
@@ -197,19 +241,18 @@ def oracle_rate(patterns, data: np.ndarray, target_s: float = 15.0, threads=None
 
 
 def run_reference(args):
+    """The CPU oracle, as it stands, on a bounded prefix of the SAME workload
+    the GPU arm times (same generator, seed and length), on this box's host
+    cores; rank 0 only."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    if args.config == "tiny":
-        pats, data, n, name = load_workload("tiny")
-    else:
-        pb, ib, n, name = WORKLOADS[args.config]
-        pats = pb()
-        data = ib(16 << 20, 0)
+    pats, data, nbytes, name = load_workload(args.config, (args.length_mib << 20) if args.length_mib else None, 0)
+    probe = data[: 1 << 16]
+    for _ in range(args.warmup):  # untimed warm-up: page in the oracle and its DFA caches
+        oracle_rate(pats, probe, target_s=0.0)
     rates = []
     samples = []
-    for _ in range(args.warmup):
-        pass
     for _ in range(max(1, args.steps)):
         r, n, dt, thr = oracle_rate(pats, data, target_s=max(2.0, 30.0 / max(1, args.steps)))
         rates.append(r)
@@ -220,9 +263,10 @@ def run_reference(args):
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": 1e3 * n / (gbs * 1e9), "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "u8", "data": "synthetic",
-            "config": {"workload": name, "n_regex": len(pats), "input_bytes": 256 << 20},
-            "cpu_baseline": {"value": gbs, "unit": "GB/s", "cores": thr, "kind": "oracle",
-                             "sample": f"all {len(pats)} regexes over the first {n} bytes of the input "
+            "config": {"workload": name, "n_regex": len(pats), "input_bytes_per_gpu": int(data.size),
+                       "parallelism": "host cores (rank 0 only)"},
+            "cpu_baseline": {"value": gbs, "unit": "GB/s", "cores": thr, "cpu": cpu_model(), "kind": "oracle",
+                             "sample": f"all {len(pats)} regexes over the first {n} bytes of the bench input "
                                        f"({dt:.1f} s per step, Thompson NFA + lazy DFA cache)"},
             "e2e": {"value": gbs, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -248,7 +292,7 @@ def main():
     ap.add_argument("--interval", type=int, default=0, help="experiment: zero-block guard interval (rx_options)")
     ap.add_argument("--split", default="chunk", choices=["chunk", "regex"], help="multi-GPU partition (N>1)")
     ap.add_argument("--ablate", default="", help="comma list of rx flags to set (ablation ladder, DESIGN.md): "
-                    "no_prefilter, modeb, no_lockstep, no_guards, rebalance")
+                    "no_prefilter, modeb, no_lockstep, lockstep_round, no_guards, rebalance")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -395,7 +439,7 @@ def main():
                                                                   else " < L2: L2 flushed between steps"),
                    "prefilter": not args.no_prefilter, "ablate": args.ablate or None, "compile_s": round(compile_s, 1),
                    **popts},
-        "roofline": roofline(ktimes, nbytes, len(pats), hbm, hbm_src, name, ms),
+        "roofline": roofline(ktimes, nbytes, len(pats), hbm, hbm_src, name, ms, args.steps),
         "clocks": clocks,
         "gpu_launches": sum(v[1] for v in ktimes.values()) or launches_per_step * args.steps,
     }
@@ -404,7 +448,7 @@ def main():
                        "d2h_bytes_per_step": 8 * len(all_pats)}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         r, n, dt, thr = oracle_rate(pats, data, target_s=15.0)
-        line["cpu_baseline"] = {"value": r, "unit": "GB/s", "cores": thr, "kind": "oracle",
+        line["cpu_baseline"] = {"value": r, "unit": "GB/s", "cores": thr, "cpu": cpu_model(), "kind": "oracle",
                                 "sample": f"all {len(pats)} regexes over the first {n} bytes ({dt:.1f} s)"}
     if rank == 0:
         print(json.dumps(line), flush=True)

@@ -83,6 +83,8 @@ typedef struct {
                                  profiles/r2_ablation_snort.md) */
 #define RX_F_NO_LOCKSTEP 128u /* sparse pass 1 without cluster lockstep: each warp runs its own windows'
                                  clusters freely (ablation) */
+#define RX_F_LOCKSTEP_ROUND 512u /* cluster lockstep with one CTA barrier per window round instead of one per
+                                   cluster (experiment) */
 #define RX_F_STATS 64u        /* debug: count visited / active windows and walk-backs per rx_match and print
                                  them to stderr (synchronises the stream; not for timing) */
 

@@ -20,7 +20,7 @@ _lib = None
 
 RX_OK, RX_EPARSE, RX_EUNSUPPORTED, RX_ETOOBIG, RX_EJIT, RX_ECUDA, RX_EINVAL, RX_ENOMEM, RX_EOVERFLOW = range(9)
 RX_F_NO_REBALANCE, RX_F_NO_GUARDS, RX_F_NO_CACHE, RX_F_REBALANCE, RX_F_NO_PREFILTER = 1, 2, 4, 8, 16
-RX_F_NO_MODEB, RX_F_STATS, RX_F_NO_LOCKSTEP, RX_F_MODEB = 32, 64, 128, 256
+RX_F_NO_MODEB, RX_F_STATS, RX_F_NO_LOCKSTEP, RX_F_MODEB, RX_F_LOCKSTEP_ROUND = 32, 64, 128, 256, 512
 
 EXPORTED = ["rx_compile", "rx_free", "rx_num_regex", "rx_num_groups", "rx_max_lookback", "rx_max_lookahead",
             "rx_boundary_bytes", "rx_program_source", "rx_program_info", "rx_match", "rx_match_chunk",

@@ -304,7 +304,8 @@ struct RxParams {
   int mode;                 // 0 = pass 1, 1 = fix-up with stored segment states, 2 = rematch
   int accumulate;           // counts/digests are added to (else the host zeroed them)
   int modeb;                // mode B allowed (plain rx_match: no chunk state in/out)
-  int lockstep;             // sparse pass 1: cluster lockstep across the CTA's warps (rx_run_segment_pf)
+  int lockstep;             // sparse pass 1 (rx_run_segment_pf): 0 free-running warps, 1 cluster lockstep
+                            // (a barrier per cluster), 2 round lockstep (a barrier per window round)
   // cross-regex prefilter (rx_prefilter_run below; rx_prefilter.cpp
   // build_prefilter documents the table blob)
   const u32 *pf_tab;
@@ -313,7 +314,8 @@ struct RxParams {
   u32 pf_o_b3, pf_o_b2, pf_o_ht, pf_o_ext, pf_o_fgoff, pf_o_fgent;
   u32 *pf_gbits;            // [NG][ntiles]: bit b of word t = a factor of the group occurs in block 32t+b
   u32 *pf_mmask;            // [NG][32*ntiles]: members whose FIRST factor occurs in the block
-  u32 *pf_omask;            // [NG][32*ntiles]: members whose OUTPUT factor occurs in the block
+  u32 *pf_omask;            // [NG][32*ntiles]: members whose OUTPUT factor occurs in the block (null: the
+                            // program has no output factor, mode B off)
                             // (both written wherever a pf_gbits bit is set)
   u32 *pf_cnt;              // [NG][32][2]: blocks with a first / output factor hit per member (mode choice)
   i64 pf_ntiles;
@@ -760,7 +762,7 @@ DEV void rx_run_segment_pf(const RxParams &p, int seg, RxOut *o, u64 *acc, u32 *
   const RxRange ir = rx_interior(p);
   const u32 *gb = p.pf_gbits + (i64)G::GID * p.pf_ntiles;
   const u32 *mmf = p.pf_mmask + (i64)G::GID * 32 * p.pf_ntiles;
-  const u32 *mmo = p.pf_omask + (i64)G::GID * 32 * p.pf_ntiles;
+  const u32 *mmo = p.pf_omask ? p.pf_omask + (i64)G::GID * 32 * p.pf_ntiles : nullptr;
   auto frame_blocks = [&](i64 w, i64 &b0, i64 &b1) {
     i64 flo = (w * Bw - Lw) * 32, fhi = flo + 1024 * K;
     if (flo < p.avail_lo) flo = p.avail_lo;
@@ -793,7 +795,8 @@ DEV void rx_run_segment_pf(const RxParams &p, int seg, RxOut *o, u64 *acc, u32 *
       const u32 word = gb[c0 >> 5];
       const i64 b = c0 + c.lane;
       bool need = false;
-      if (((word >> c.lane) & 1u) && b >= b0 && b <= bmax) need = ((mmf[b] & ~bm) | (mmo[b] & bm)) != 0u;
+      if (((word >> c.lane) & 1u) && b >= b0 && b <= bmax)
+        need = ((mmf[b] & ~bm) | (bm ? (mmo[b] & bm) : 0u)) != 0u;
       const u32 bal = __ballot_sync(RX_FULL, need);
       if (!bal) continue;
       const i64 bb = c0 + (__ffs(bal) - 1);
@@ -852,7 +855,7 @@ DEV void rx_run_segment_pf(const RxParams &p, int seg, RxOut *o, u64 *acc, u32 *
       for (i64 b = b0 + c.lane; b <= b1; b += 32)
         if ((gb[b >> 5] >> (b & 31)) & 1u) {
           fmine |= mmf[b];
-          omine |= mmo[b];
+          if (mmo) omine |= mmo[b];
         }
       const u32 fm = __reduce_or_sync(RX_FULL, fmine), om = __reduce_or_sync(RX_FULL, omine);
       const u32 rmask = (fm & ~bm) | (om & bm);
@@ -928,7 +931,7 @@ DEV void rx_run_segment_pf(const RxParams &p, int seg, RxOut *o, u64 *acc, u32 *
         U = 0u;
       }
       if (m) G::body_i(c, pl, st, nst, m);
-      if (lock) __syncthreads();
+      if (lock && p.lockstep == 1) __syncthreads();  // 2: one barrier per round only
     }
     if (!have) continue;
     u32 *t = st;
@@ -1239,6 +1242,9 @@ DEV void rx_prefilter_run(const RxParams &p, int NG) {
                  ? __ldg(reinterpret_cast<const u32 *>(p.in + base - 4))
                  : rx_load_u32_slow(p, base - 4);
       // filter pass over the 16 positions -> hit masks per anchor length
+      // (measured: gating the Bloom tests behind a trailing-bigram bitmap
+      // made the kernel slower -- most text positions pass the gate and the
+      // gated loop runs divergent, profiles/r2_ncu_r2k*)
       u32 h4 = 0u, h3 = 0u, h2 = 0u;
 #pragma unroll
       for (int r = 0; r < 16; ++r) {
@@ -1283,7 +1289,7 @@ DEV void rx_prefilter_run(const RxParams &p, int NG) {
       if (lane == 0) p.pf_gbits[(i64)g * p.pf_ntiles + t] = bal;
       if (f | o) {
         p.pf_mmask[(i64)g * nblk + t * 32 + lane] = f;
-        p.pf_omask[(i64)g * nblk + t * 32 + lane] = o;
+        if (p.pf_omask) p.pf_omask[(i64)g * nblk + t * 32 + lane] = o;
       }
       if (bal && p.pf_cnt) {
         u32 cf = 0u, co = 0u;

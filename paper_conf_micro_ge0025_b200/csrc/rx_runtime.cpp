@@ -211,7 +211,7 @@ constexpr size_t kPfTagBytes = 4 * 32 * 64;  // prefilter factor tags (RX_PF_TAG
 constexpr size_t kCtaHdr = 512;  // CTA header of pass 1 / fix-up shared memory (RX_CTA_HDR, rx_device.cuh)
 constexpr int kPrefilterWarps = 8;
 constexpr size_t kMaxSmem = 232448;  // opt-in dynamic shared memory per block (227 KB)
-constexpr size_t kModuleBytes = 48u << 20;  // code per linked module (see rx_compile)
+constexpr size_t kModuleBytes = 128u << 20;  // code per linked module (see rx_compile)
 struct RxModule {
   int g_begin = 0, g_end = 0;  // group range
   int ns_max = 1, nr_max = 1;
@@ -588,7 +588,13 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
     p->all_source += ksrc[m];
     p->mods.push_back(std::move(mod));
   }
-  p->info += "modules: " + std::to_string(ranges.size()) + "\n";
+  p->info += "modules: " + std::to_string(ranges.size()) + " (code MB:";
+  for (auto &m : p->mods) {
+    size_t b = 0;
+    for (auto &u : m.units) b += u.size();
+    p->info += " " + std::to_string(b >> 20);
+  }
+  p->info += ")\n";
   *out = p;
   return RX_OK;
 }
@@ -780,7 +786,7 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
   // stream: its walk-back may read any earlier byte and reconstructs state
   // from the stream start, so chunks (incoming / outgoing state) use mode A
   prm.modeb = (mode == 0 && !st_in && !st_out && halo_left == 0) ? 1 : 0;
-  prm.lockstep = (p->flags & RX_F_NO_LOCKSTEP) ? 0 : 1;
+  prm.lockstep = (p->flags & RX_F_NO_LOCKSTEP) ? 0 : ((p->flags & RX_F_LOCKSTEP_ROUND) ? 2 : 1);
   if (!prm.status) {
     unsigned int *status_scratch = (unsigned int *)scratch_get(p, stream, SC_STATUS, 256);
     if (!status_scratch) return fail(RX_ENOMEM, "status");
@@ -839,7 +845,11 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
     const size_t gb_bytes = ((size_t)4 * (size_t)ntiles * (size_t)G + 255) & ~(size_t)255;
     const size_t bl_bytes = ((size_t)4 * 32 * (size_t)ntiles * (size_t)G + 255) & ~(size_t)255;
     const size_t cnt_bytes = (size_t)4 * 64 * (size_t)G;
-    char *pf_scratch = (char *)scratch_get(p, stream, SC_PF, gb_bytes + 2 * bl_bytes + cnt_bytes + 256);
+    // output-factor masks only if some regex has output factors (mode B)
+    bool any_out = false;
+    for (auto &rf : p->cs.rf) any_out = any_out || !rf.out.empty();
+    const size_t ob_bytes = any_out ? bl_bytes : 0;
+    char *pf_scratch = (char *)scratch_get(p, stream, SC_PF, gb_bytes + bl_bytes + ob_bytes + cnt_bytes + 256);
     if (!pf_scratch) return fail(RX_ENOMEM, "prefilter scratch");
     const rx::Prefilter &pf = p->cs.pf;
     RxModule &m0 = p->mods[0];
@@ -857,11 +867,13 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
     prm.pf_o_fgent = pf.o_fgent;
     prm.pf_gbits = (unsigned int *)pf_scratch;
     prm.pf_mmask = (unsigned int *)(pf_scratch + gb_bytes);
-    prm.pf_omask = (unsigned int *)(pf_scratch + gb_bytes + bl_bytes);
-    prm.pf_cnt = (unsigned int *)(pf_scratch + gb_bytes + 2 * bl_bytes);
+    prm.pf_omask = any_out ? (unsigned int *)(pf_scratch + gb_bytes + bl_bytes) : nullptr;
+    // per-member block counts feed only the mode-B choice
+    prm.pf_cnt = any_out ? (unsigned int *)(pf_scratch + gb_bytes + bl_bytes + ob_bytes) : nullptr;
     prm.pf_ntiles = ntiles;
     prm.pf_on = 1;
-    if (cudaMemsetAsync(prm.pf_cnt, 0, cnt_bytes, stream) != cudaSuccess) return fail(RX_ECUDA, "memset");
+    if (prm.pf_cnt && cudaMemsetAsync(prm.pf_cnt, 0, cnt_bytes, stream) != cudaSuccess)
+      return fail(RX_ECUDA, "memset");
     // 8-warp CTAs, several per SM (the verification of filter hits is a
     // chain of dependent loads: more resident warps hide it)
     s = launch(p, m0, m0.prefilter, std::min<long long>(ntiles, 148LL * 8), kPrefilterWarps, prm, stream);

@@ -32,6 +32,11 @@ CFG = {
                 "dotstar/protomata-like 2k regexes x 1 GiB"),
     # config 5: all 10k regexes over a 64 MiB sample of the 8 GiB multi input
     # (the first 16 MiB of each of its four 2 GiB family parts, concatenated)
+    # config 5 as the GPU tests build it in seconds: the 64 MiB multi stream
+    # (four 16 MiB family parts, gen.multi_input(64 MiB)); the 8 GiB test
+    # tiles it (tests/test_gpu_config5.py)
+    "multi64": (lambda: gen.multi_patterns(2500), lambda: gen.multi_input(64 << 20, seed=5),
+                "multi 10k regexes x 64 MiB (gen.multi_input(64 MiB, seed 5): four 16 MiB family parts)"),
     "multi64m": (lambda: gen.multi_patterns(2500), lambda: multi_sample(),
                  "multi 10k regexes x 64 MiB sample (first 16 MiB of each 2 GiB part of the 8 GiB input)"),
 }
