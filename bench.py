@@ -290,6 +290,8 @@ def main():
     ap.add_argument("--max-regs", type=int, default=0, help="experiment: registers per thread (rx_options; "
                     "pass-1 CTA = 64K / (32 x max_regs) warps)")
     ap.add_argument("--interval", type=int, default=0, help="experiment: zero-block guard interval (rx_options)")
+    ap.add_argument("--batch", type=int, default=0, help="N3: match N independent packet-sized records (0-1460 B, "
+                    "cut from the workload's input) with rx_match_batch, one launch sequence per step")
     ap.add_argument("--split", default="chunk", choices=["chunk", "regex"], help="multi-GPU partition (N>1)")
     ap.add_argument("--ablate", default="", help="comma list of rx flags to set (ablation ladder, DESIGN.md): "
                     "no_prefilter, modeb, no_lockstep, lockstep_round, no_guards, rebalance")
@@ -344,9 +346,32 @@ def main():
     def step_device():
         prog.match(d_in, out=out, stream=stream)
 
+    if args.batch:
+        # N3: records of 0-1460 B (seeded), back to back from the input start
+        rng = np.random.default_rng(1460)
+        lens = rng.integers(0, 1461, size=args.batch)
+        offs = np.concatenate([[0], np.cumsum(lens)]).astype(np.uint64)
+        assert int(offs[-1]) <= nbytes, "input too short for that many records"
+        nbytes = int(offs[-1])
+        d_batch = d_in[:nbytes]
+        bout = prog.match_batch(d_batch, offs, digests=False, stream=stream)
+        name = f"{name}; rx_match_batch of {args.batch} records (0-1460 B)"
+
+        def step_device():  # noqa: F811
+            prog.match_batch(d_batch, offs, stream=stream, out=bout)
+
     def step_e2e():
         # the public API end to end: H2D of the step's input from pinned host
-        # memory, the step (with its collectives at N > 1), D2H of the counts
+        # memory, the step (with its collectives at N > 1), D2H of the counts.
+        # At N = 1 through rx_match_host, which overlaps the copy of piece i+1
+        # with the matching of piece i (exact: pieces in order, state chained)
+        if args.batch:
+            d_in[:nbytes].copy_(host[:nbytes], non_blocking=True)
+            step_device()
+            return bout["counts"].to("cpu", non_blocking=False)
+        if world == 1:
+            prog.match_host(host, out=out, stream=stream, device=dev)
+            return out["counts"].to("cpu", non_blocking=False)
         d_in.copy_(host, non_blocking=True)
         step_device()
         return (full if split_regex else out["counts"]).to("cpu", non_blocking=False)
@@ -445,7 +470,10 @@ def main():
     }
     if e2e_ms is not None:
         line["e2e"] = {"value": total_bytes / (e2e_ms * 1e-3) / 1e9, "unit": "GB/s", "h2d_bytes_per_step": nbytes,
-                       "d2h_bytes_per_step": 8 * len(all_pats)}
+                       "d2h_bytes_per_step": 8 * len(all_pats) * (args.batch or 1),
+                       "api": ("H2D copy + rx_match_batch" if args.batch else
+                               "rx_match_host (pinned host input, pipelined 32 MiB pieces)") if world == 1
+                       else "H2D copy + rx_match_chunk protocol"}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         r, n, dt, thr = oracle_rate(pats, data, target_s=15.0)
         line["cpu_baseline"] = {"value": r, "unit": "GB/s", "cores": thr, "cpu": cpu_model(), "kind": "oracle",

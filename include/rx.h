@@ -184,6 +184,23 @@ rx_status rx_rematch_chunk(const rx_program *p, const uint8_t *d_input, uint64_t
 rx_status rx_match_batch(const rx_program *p, const uint8_t *d_input, const uint64_t *offsets, uint32_t n_streams,
                          void *stream, const rx_output *out);
 
+/* Whole stream from HOST memory, end to end: the input is copied to the
+ * device in pieces of piece_bytes (0 = 32 MiB; rounded up to a multiple of
+ * 1 KiB) on an internal copy stream, and piece i is matched with
+ * rx_match_chunk while piece i+1 is in flight.  Pieces are matched in order on
+ * `stream`, each with rx_max_lookback bytes of the previous piece as its left
+ * halo, rx_max_lookahead bytes of the next as its right halo and the previous
+ * piece's end state as its exact incoming state, so the result equals
+ * rx_match over the whole stream (counts, digests, match list; dense words
+ * at their stream positions).  h_input should be page-locked (cudaHostAlloc /
+ * cudaHostRegister) for the copies to overlap; pageable memory works but
+ * serialises them.  Device staging buffers are owned by the program (reused
+ * call after call).  Outputs are OVERWRITTEN.  Asynchronous on `stream`:
+ * h_input must stay valid and unmodified until the stream reaches the end of
+ * the call's work.  Errors as rx_match, RX_ENOMEM for the staging buffers. */
+rx_status rx_match_host(const rx_program *p, const uint8_t *h_input, uint64_t len, uint64_t piece_bytes, void *stream,
+                        const rx_output *out);
+
 /* Per-kernel device timing (for roofline reporting): when on, every launch
  * of the program is bracketed by CUDA events on its stream.  rx_kernel_times
  * waits for the recorded events and writes the accumulated milliseconds and

@@ -25,7 +25,7 @@ RX_F_NO_MODEB, RX_F_STATS, RX_F_NO_LOCKSTEP, RX_F_MODEB, RX_F_LOCKSTEP_ROUND = 3
 EXPORTED = ["rx_compile", "rx_free", "rx_num_regex", "rx_num_groups", "rx_max_lookback", "rx_max_lookahead",
             "rx_boundary_bytes", "rx_program_source", "rx_program_info", "rx_match", "rx_match_chunk",
             "rx_rematch_chunk", "rx_last_error", "rx_kernels_per_match", "rx_set_profiling", "rx_kernel_times", "rx_match_batch",
-            "rx_prefilter_table"]
+            "rx_prefilter_table", "rx_match_host"]
 
 
 class RxError(RuntimeError):
@@ -87,6 +87,8 @@ def load_library():
         lib.rx_rematch_chunk.restype = ctypes.c_int
         lib.rx_match_batch.argtypes = [vp, vp, vp, u32, vp, ctypes.POINTER(_Output)]
         lib.rx_match_batch.restype = ctypes.c_int
+        lib.rx_match_host.argtypes = [vp, vp, u64, u64, vp, ctypes.POINTER(_Output)]
+        lib.rx_match_host.restype = ctypes.c_int
         lib.rx_set_profiling.argtypes = [vp, ctypes.c_int]
         lib.rx_set_profiling.restype = ctypes.c_int
         lib.rx_kernel_times.argtypes = [vp, vp, vp, ctypes.c_int]
@@ -271,7 +273,21 @@ class Program:
                                           ctypes.byref(s)))
         return out
 
-    def match_batch(self, data, offsets, dense=False, digests=True, match_cap=None, stream=None):
+    def match_host(self, host, out=None, piece_bytes=0, dense=False, digests=True, match_cap=None, stream=None,
+                   device=None):
+        """rx_match_host: `host` a CPU uint8 tensor (pin_memory() for overlap);
+        pipelined host-to-device copy + matching, result as match()."""
+        import torch
+        assert host.device.type == "cpu" and host.dtype == torch.uint8 and host.is_contiguous()
+        device = device or torch.device("cuda", torch.cuda.current_device())
+        if out is None:
+            out = self.alloc_outputs(host.numel(), device, dense=dense, digests=digests, match_cap=match_cap)
+        s = self._out_struct(out)
+        _check(self._lib.rx_match_host(self._h, ctypes.c_void_p(host.data_ptr() if host.numel() else None),
+                                       int(host.numel()), int(piece_bytes), _stream_handle(stream), ctypes.byref(s)))
+        return out
+
+    def match_batch(self, data, offsets, dense=False, digests=True, match_cap=None, stream=None, out=None):
         """rx_match_batch: `data` a CUDA uint8 tensor holding the streams back
         to back, `offsets` n_streams + 1 host ints.  Returns counts
         int64[n_streams, n_regex], digests int64[n_streams, n_regex, 2] (over
@@ -284,8 +300,14 @@ class Program:
         ns = max(len(offs) - 1, 0)
         n, dev = self.n_regex, data.device
         max_len = int((offs[1:] - offs[:-1]).max()) if ns else 0
+        if out is not None:  # reuse the buffers of an earlier call with the same shape
+            s = self._out_struct(out)
+            s.d_counts = out["counts_full"].data_ptr()
+            _check(self._lib.rx_match_batch(self._h, _ptr(data), offs.ctypes.data_as(ctypes.c_void_p), ns,
+                                            _stream_handle(stream), ctypes.byref(s)))
+            return out
         counts_full = torch.zeros((max(ns, 1), max(n, 1)), dtype=torch.int64, device=dev)
-        out = {"counts": counts_full[:ns, :n],
+        out = {"counts": counts_full[:ns, :n], "counts_full": counts_full,
                "digests": torch.zeros((max(ns, 1), max(n, 1), 2), dtype=torch.int64, device=dev)[:ns, :n]
                if digests else None,
                "status": torch.zeros(1, dtype=torch.int32, device=dev)}

@@ -622,17 +622,21 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
   //   | window staging [TB] (TMA) | mbarrier u64
   const int LB = lit_scratch_bytes(cs), TB = 1024 * max_words_per_lane(cs);
   const int ACC = (24 * nrmax + 15) & ~15, OUTB = 96, STB = ((24 * nsmax) + 15) & ~15;
-  const int PER = ACC + OUTB + STB + LB + TB + 16;
+  const int PER = ACC + OUTB + STB + LB + TB + 16 + 512;  // + per-warp parameter copy (rx_match_batch)
   os << "static_assert(sizeof(RxOut) <= " << OUTB << ", \"RxOut layout\");\n";
   os << "#define RX_WARP_SMEM_" << gi << " " << PER << "\n";
   // The launch parameters are read from the CTA header of the dynamic shared
   // memory (rx_cta_params, copied there by the kernel): a reference to the
   // kernel parameter handed across this out-of-line call made every field
   // read a generic load through a spilled pointer (profiles/r2_*).
-  os << "extern \"C\" __device__ __noinline__ void rx_seg_" << gi << "(int seg) {\n"
-     << "  const RxParams &p = rx_cta_params();\n"
+  os << "extern \"C\" __device__ __noinline__ void rx_seg_" << gi << "(int seg_in) {\n"
+     << "  const RxParams &pc = rx_cta_params();\n"
      << "  const int warp = threadIdx.x >> 5;\n"
      << "  unsigned char *base = rx_warp_smem(warp, " << PER << ");\n"
+     << "  RxParams *wp = reinterpret_cast<RxParams *>(base + " << PER - 512 << ");\n"
+     << "  const bool batch = pc.batch_off != nullptr;\n"
+     << "  const RxParams &p = batch ? rx_batch_view(pc, wp, seg_in, " << (int)cs.irs.size() << ") : pc;\n"
+     << "  const int seg = batch ? 0 : seg_in;\n"
      << "  u64 *acc = reinterpret_cast<u64 *>(base);\n"
      << "  RxOut *o = reinterpret_cast<RxOut *>(base + " << ACC << ");\n"
      << "  u32 *st = reinterpret_cast<u32 *>(base + " << ACC + OUTB << ");\n"
@@ -659,7 +663,7 @@ size_t warp_smem_bytes(const CompiledSet &cs) {
   int nsmax, nrmax;
   layout(cs, nsmax, nrmax);
   const int LB = lit_scratch_bytes(cs), TB = 1024 * max_words_per_lane(cs);
-  return (size_t)(((24 * nrmax + 15) & ~15) + 96 + (((24 * nsmax) + 15) & ~15) + LB + TB + 16);
+  return (size_t)(((24 * nrmax + 15) & ~15) + 96 + (((24 * nsmax) + 15) & ~15) + LB + TB + 16 + 512);
 }
 
 // The kernel unit: rx_pass1 (a CTA of 16 warps runs one group over 16

@@ -327,6 +327,12 @@ struct RxParams {
   int fix_phase;            // mode 1: 1 = parallel per segment, 2 = serial remainder
   u32 *seg_fix;             // [nseg_max][G][NSMAX]: phase-1 end state of a segment that did not converge
   u32 *seg_nc;              // [nseg_max][G]: that segment did not converge in phase 1
+  // rx_match_batch (one launch sequence for all streams): stream s is
+  // in[batch_off[s] .. batch_off[s+1]); pass-1 "segment" s = stream s, whose
+  // warp runs it whole with its own copy of these parameters (rx_batch_view)
+  const u64 *batch_off;     // device u64[batch_n + 1] (null: not a batch)
+  i64 batch_n;
+  i64 pf_shift;             // prefilter block coordinates = stream position + pf_shift
 };
 
 // CTA header of the dynamic shared memory (pass 1 and fix-up): the launch
@@ -346,6 +352,41 @@ DEV void rx_cta_params_store(const RxParams &p) {
   u32 *dst = reinterpret_cast<u32 *>(rx_dyn_smem());
   for (int i = threadIdx.x; i < (int)(sizeof(RxParams) / 4); i += blockDim.x) dst[i] = src[i];
   __syncthreads();
+}
+
+// rx_match_batch: this warp's stream s as a whole input of its own (zero
+// state in, nothing readable outside it), written over a per-warp copy of the
+// launch parameters; warps beyond the last stream get an empty stream (they
+// still take part in the CTA's lockstep barriers)
+DEV const RxParams &rx_batch_view(const RxParams &pc, RxParams *wp, i64 s, int nreg) {
+  const u32 lane = threadIdx.x & 31u;
+  const u32 *src = reinterpret_cast<const u32 *>(&pc);
+  u32 *dst = reinterpret_cast<u32 *>(wp);
+  for (int i = (int)lane; i < (int)(sizeof(RxParams) / 4); i += 32) dst[i] = src[i];
+  __syncwarp();
+  if (lane == 0) {
+    const bool ok = s < pc.batch_n;
+    const u64 o0 = ok ? pc.batch_off[s] : 0ull, o1 = ok ? pc.batch_off[s + 1] : 0ull;
+    const i64 len = (i64)(o1 - o0);
+    wp->in = pc.in + o0;
+    wp->avail_lo = wp->valid_lo = 0;
+    wp->avail_hi = wp->valid_hi = wp->len = len;
+    wp->gofs = pc.gofs + (i64)o0;
+    wp->pf_shift = (i64)o0;
+    const i64 ss = ok ? s : 0;
+    wp->counts = pc.counts + ss * nreg;
+    wp->digests = pc.digests ? pc.digests + 2 * ss * nreg : nullptr;
+    wp->dense = pc.dense ? pc.dense + (u64)ss * nreg * pc.pitch : nullptr;
+    wp->aligned = ((reinterpret_cast<unsigned long long>(wp->in) & 15ull) == 0ull) ? 1 : 0;
+    wp->sw = 1 << 30;
+    wp->nseg_max = 1;
+    wp->seg_state = nullptr;
+    wp->st_in = nullptr;
+    wp->st_out = nullptr;
+    wp->modeb = 0;
+  }
+  __syncwarp();
+  return *wp;
 }
 
 // split prologue (software pipelining): rx_fetch issues the 128-bit loads of
@@ -605,7 +646,7 @@ DEV void rx_run_segment_dense(const RxParams &p, int seg, RxOut *o, u64 *acc, u3
     __syncthreads();
   }
   if (!live) return;
-  if (NS > 0) {
+  if (NS > 0 && p.seg_state) {
     u32 *dst = p.seg_state + ((i64)seg * G::NG + G::GID) * G::NSMAX;
     for (int s = (int)c.lane; s < NS; s += 32) dst[s] = st[s];
     if (p.st_out && w_end == nwin)
@@ -768,8 +809,8 @@ DEV void rx_run_segment_pf(const RxParams &p, int seg, RxOut *o, u64 *acc, u32 *
     if (flo < p.avail_lo) flo = p.avail_lo;
     if (fhi > p.avail_hi) fhi = p.avail_hi;
     if (fhi <= flo) fhi = flo + 1;
-    b0 = (flo - p.avail_lo) >> 10;
-    b1 = (fhi - 1 - p.avail_lo) >> 10;
+    b0 = (flo - p.avail_lo + p.pf_shift) >> 10;
+    b1 = (fhi - 1 - p.avail_lo + p.pf_shift) >> 10;
   };
   i64 bmax = 0;
   if (w_begin < w_end) {
@@ -801,7 +842,7 @@ DEV void rx_run_segment_pf(const RxParams &p, int seg, RxOut *o, u64 *acc, u32 *
       if (!bal) continue;
       const i64 bb = c0 + (__ffs(bal) - 1);
       if (bb <= b1) return w;
-      const i64 pos = p.avail_lo + bb * RX_PF_BLK;
+      const i64 pos = p.avail_lo + bb * RX_PF_BLK - p.pf_shift;
       const i64 wn = rx_floor_div(rx_floor_div(pos, 32) + Lw - 32 * K, Bw) + 1;
       const i64 r = wn > w + 1 ? wn : w + 1;
       return r < w_end ? r : w_end;
@@ -945,7 +986,7 @@ DEV void rx_run_segment_pf(const RxParams &p, int seg, RxOut *o, u64 *acc, u32 *
   }
   if (staged >= 0) retire();
   if (!live) return;
-  if (NS > 0) {
+  if (NS > 0 && p.seg_state) {
     // mode-B slots are not carried across segments (the next segment walks
     // back for itself): the fix-up sees zero for them on both sides
     u32 *dst = p.seg_state + ((i64)seg * G::NG + G::GID) * G::NSMAX;

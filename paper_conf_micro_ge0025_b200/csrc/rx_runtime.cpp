@@ -252,11 +252,21 @@ struct rx_program {
   // cudaMallocAsync/cudaFreeAsync pair per buffer per call left the GPU idle
   // between steps (7.5 ms per Snort-like step, 55 ms per Dotstar-like step)
   std::map<std::pair<void *, int>, std::pair<void *, size_t>> scratch;
+  // rx_match_host: copy stream, staging ring and its events (lazily created)
+  cudaStream_t copy_stream = nullptr;
+  static constexpr int kRing = 3;
+  void *ring[kRing] = {nullptr, nullptr, nullptr};
+  size_t ring_bytes = 0;
+  cudaEvent_t copied[kRing] = {nullptr, nullptr, nullptr}, consumed[kRing] = {nullptr, nullptr, nullptr};
+  void *states[2] = {nullptr, nullptr};
+  // rx_match_batch: pinned staging of the stream offsets
+  void *batch_host = nullptr;
+  size_t batch_host_bytes = 0;
 };
 
 namespace {
 // scratch slots of one rx_match call
-enum { SC_STATUS = 0, SC_SEGSTATE = 1, SC_PF = 2, SC_FIX = 3 };
+enum { SC_STATUS = 0, SC_SEGSTATE = 1, SC_PF = 2, SC_FIX = 3, SC_BATCH = 4 };
 void *scratch_get(rx_program *p, cudaStream_t s, int slot, size_t bytes) {
   std::lock_guard<std::mutex> lk(p->mu);
   auto &e = p->scratch[{(void *)s, slot}];
@@ -347,6 +357,15 @@ void rx_free(rx_program *p) {
     }
   for (auto &kv : p->scratch)
     if (kv.second.first) cudaFree(kv.second.first);
+  for (int i = 0; i < rx_program::kRing; ++i) {
+    if (p->ring[i]) cudaFree(p->ring[i]);
+    if (p->copied[i]) cudaEventDestroy(p->copied[i]);
+    if (p->consumed[i]) cudaEventDestroy(p->consumed[i]);
+  }
+  for (int i = 0; i < 2; ++i)
+    if (p->states[i]) cudaFree(p->states[i]);
+  if (p->copy_stream) cudaStreamDestroy(p->copy_stream);
+  if (p->batch_host) cudaFreeHost(p->batch_host);
   delete p;
 }
 
@@ -645,6 +664,9 @@ struct RxParamsHost {  // must mirror RxParams in rx_device.cuh (tests/test_libr
   int fix_phase;
   unsigned int *seg_fix;
   unsigned int *seg_nc;
+  const unsigned long long *batch_off;
+  long long batch_n;
+  long long pf_shift;
 };
 
 rx_status ensure_loaded(rx_program *p, int &device) {
@@ -734,9 +756,17 @@ rx_status launch(rx_program *p, RxModule &m, CUfunction f, long long blocks, int
 
 long long div_up(long long a, long long b) { return (a + b - 1) / b; }
 
+// batch: rx_match_batch -- d_input/len span all streams back to back, the
+// per-stream outputs are laid out by stream, `batch_off` (device) holds the
+// n_streams + 1 offsets; one launch sequence for all streams
+struct BatchArg {
+  const unsigned long long *d_off;
+  long long n;
+};
+
 rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo_left, uint64_t halo_right,
               uint64_t gofs, const void *st_in, void *st_out, const void *st_assumed, int accumulate, int mode,
-              cudaStream_t stream, const rx_output *out) {
+              cudaStream_t stream, const rx_output *out, const BatchArg *batch = nullptr) {
   if (!p || !out || !out->d_counts) return fail(RX_EINVAL, "null argument");
   if (len && !d_input) return fail(RX_EINVAL, "null input");
   if (out->d_bitstreams && out->pitch_words < (len + 31) / 32) return fail(RX_EINVAL, "pitch_words too small");
@@ -817,6 +847,14 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
   const long long cpg0 = std::max<long long>(1, div_up(target_ctas, std::max(G, 1)));
   long long sw = std::max<long long>(4, div_up(max_nwin, cpg0 * p->pass1_warps));
   long long nseg_max = std::max<long long>(1, div_up(max_nwin, sw));
+  if (batch) {
+    // pass-1 "segment" s = stream s (one warp runs it whole: no fix-up)
+    sw = 1 << 30;
+    nseg_max = std::max<long long>(1, batch->n);
+    prm.batch_off = batch->d_off;
+    prm.batch_n = batch->n;
+    prm.modeb = 0;
+  }
   const long long cpg = div_up(nseg_max, p->pass1_warps);
   prm.sw = (int)std::min<long long>(sw, 1 << 30);
   prm.nseg_max = (int)nseg_max;
@@ -832,6 +870,7 @@ rx_status run(rx_program *p, const uint8_t *d_input, uint64_t len, uint64_t halo
   }
   const size_t bytes = 4ull * (size_t)nseg_max * (size_t)G * (size_t)ns_all;
   unsigned int *seg_state = nullptr;
+  if (batch) any_state = false;  // whole streams per warp: nothing to fix up
   if (any_state && !(seg_state = (unsigned int *)scratch_get(p, stream, SC_SEGSTATE, bytes)))
     return fail(RX_ENOMEM, "seg_state");
   prm.seg_state = seg_state;
@@ -958,8 +997,10 @@ rx_status rx_rematch_chunk(const rx_program *p, const uint8_t *d_input, uint64_t
 // SURVEY 8(f) N3 / P:L178 (MIMD: many independent input streams).  Stream i
 // is d_input[offsets[i] .. offsets[i+1]) and is matched as a whole input of
 // its own (zero state at its start, nothing readable past either end), so
-// no match and no state crosses a stream boundary.  This first form issues
-// one rx_match_chunk sequence per stream on `stream`; outputs are per stream.
+// no match and no state crosses a stream boundary.  One launch sequence for
+// the whole batch: one prefilter pass over the concatenation (a factor
+// straddling two streams is only a false positive), then pass 1 with one
+// warp per (group, stream) running the stream whole (rx_batch_view).
 rx_status rx_match_batch(const rx_program *p, const uint8_t *d_input, const uint64_t *offsets, uint32_t n_streams,
                          void *stream, const rx_output *out) {
   if (!p || !out || !out->d_counts || (n_streams && !offsets)) return fail(RX_EINVAL, "null argument");
@@ -969,6 +1010,7 @@ rx_status rx_match_batch(const rx_program *p, const uint8_t *d_input, const uint
     max_len = std::max<uint64_t>(max_len, offsets[i + 1] - offsets[i]);
   }
   if (out->d_bitstreams && out->pitch_words < (max_len + 31) / 32) return fail(RX_EINVAL, "pitch_words too small");
+  if (n_streams && offsets[n_streams] && !d_input) return fail(RX_EINVAL, "null input");
   cudaStream_t st = (cudaStream_t)stream;
   const uint64_t n = p->n_regex;
   const uint64_t ns = n_streams;
@@ -981,16 +1023,92 @@ rx_status rx_match_batch(const rx_program *p, const uint8_t *d_input, const uint
   if (out->d_status && cudaMemsetAsync(out->d_status, 0, 4, st) != cudaSuccess) return fail(RX_ECUDA, "memset");
   if (out->d_match_total && cudaMemsetAsync(out->d_match_total, 0, 8, st) != cudaSuccess)
     return fail(RX_ECUDA, "memset");
-  for (uint32_t i = 0; i < n_streams; i++) {
+  if (!ns) return RX_OK;
+  const uint64_t total = offsets[ns] - offsets[0];
+  // the offsets, rebased to offsets[0], on the device (stream-ordered copy
+  // from a program-owned pinned staging buffer)
+  rx_program *pm = const_cast<rx_program *>(p);
+  const size_t obytes = 8ull * (ns + 1);
+  unsigned long long *d_off = (unsigned long long *)scratch_get(pm, st, SC_BATCH, obytes);
+  if (!d_off) return fail(RX_ENOMEM, "batch offsets");
+  unsigned long long *h_off = nullptr;
+  {
+    std::lock_guard<std::mutex> lk(pm->mu);
+    if (pm->batch_host_bytes < obytes) {
+      if (pm->batch_host) {
+        cudaStreamSynchronize(st);
+        cudaFreeHost(pm->batch_host);
+      }
+      pm->batch_host = nullptr;
+      pm->batch_host_bytes = 0;
+      if (cudaMallocHost(&pm->batch_host, obytes) != cudaSuccess) return fail(RX_ENOMEM, "batch offsets (host)");
+      pm->batch_host_bytes = obytes;
+    } else {
+      cudaStreamSynchronize(st);  // the previous batch's copy has read the staging buffer
+    }
+    h_off = (unsigned long long *)pm->batch_host;
+  }
+  for (uint64_t i = 0; i <= ns; ++i) h_off[i] = offsets[i] - offsets[0];
+  if (cudaMemcpyAsync(d_off, h_off, obytes, cudaMemcpyHostToDevice, st) != cudaSuccess)
+    return fail(RX_ECUDA, "offsets copy");
+  BatchArg b{d_off, (long long)ns};
+  // the streams' match-list positions and digests are relative to d_input
+  return run(pm, d_input + offsets[0], total, 0, 0, offsets[0], nullptr, nullptr, nullptr, 1, 0, st, out, &b);
+}
+
+rx_status rx_match_host(const rx_program *pc, const uint8_t *h_input, uint64_t len, uint64_t piece_bytes,
+                        void *stream, const rx_output *out) {
+  rx_program *p = const_cast<rx_program *>(pc);
+  if (!p || !out || !out->d_counts) return fail(RX_EINVAL, "null argument");
+  if (len && !h_input) return fail(RX_EINVAL, "null input");
+  if (out->d_bitstreams && out->pitch_words < (len + 31) / 32) return fail(RX_EINVAL, "pitch_words too small");
+  uint64_t P = piece_bytes ? piece_bytes : (32ull << 20);
+  P = (P + 1023) & ~1023ull;
+  const uint64_t hl = p->lookback, hr = p->lookahead;
+  const size_t need = (size_t)(P + hl + hr + 64);
+  const size_t sbytes = std::max<size_t>(4, 4 * (size_t)p->state_words);
+  cudaStream_t s = (cudaStream_t)stream;
+  {
+    std::lock_guard<std::mutex> lk(p->mu);
+    if (!p->copy_stream && cudaStreamCreateWithFlags(&p->copy_stream, cudaStreamNonBlocking) != cudaSuccess)
+      return fail(RX_ECUDA, "copy stream");
+    if (p->ring_bytes < need) {
+      cudaDeviceSynchronize();  // growth only
+      for (int i = 0; i < rx_program::kRing; ++i) {
+        if (p->ring[i]) cudaFree(p->ring[i]);
+        p->ring[i] = nullptr;
+        if (cudaMalloc(&p->ring[i], need) != cudaSuccess) return fail(RX_ENOMEM, "staging buffers");
+        if (!p->copied[i] && (cudaEventCreateWithFlags(&p->copied[i], cudaEventDisableTiming) != cudaSuccess ||
+                              cudaEventCreateWithFlags(&p->consumed[i], cudaEventDisableTiming) != cudaSuccess))
+          return fail(RX_ECUDA, "events");
+      }
+      p->ring_bytes = need;
+    }
+    for (int i = 0; i < 2; ++i)
+      if (!p->states[i] && cudaMalloc(&p->states[i], sbytes) != cudaSuccess) return fail(RX_ENOMEM, "state buffers");
+  }
+  if (len == 0) return rx_match(p, nullptr, 0, stream, out);
+  const uint64_t npieces = (len + P - 1) / P;
+  for (uint64_t i = 0; i < npieces; ++i) {
+    const int b = (int)(i % rx_program::kRing);
+    const uint64_t a = i * P, e = std::min(len, a + P);
+    const uint64_t lo = a >= hl ? a - hl : 0, hi = std::min(len, e + hr);
+    // the copy into ring slot b waits until the match that last read it is done
+    if (i >= (uint64_t)rx_program::kRing && cudaStreamWaitEvent(p->copy_stream, p->consumed[b], 0) != cudaSuccess)
+      return fail(RX_ECUDA, "wait");
+    if (cudaMemcpyAsync(p->ring[b], h_input + lo, hi - lo, cudaMemcpyHostToDevice, p->copy_stream) != cudaSuccess)
+      return fail(RX_ECUDA, "host-to-device copy");
+    if (cudaEventRecord(p->copied[b], p->copy_stream) != cudaSuccess ||
+        cudaStreamWaitEvent(s, p->copied[b], 0) != cudaSuccess)
+      return fail(RX_ECUDA, "event");
     rx_output o = *out;
-    o.d_counts = out->d_counts + (uint64_t)i * n;
-    if (out->d_digests) o.d_digests = out->d_digests + 2ull * i * n;
-    if (out->d_bitstreams) o.d_bitstreams = out->d_bitstreams + (uint64_t)i * n * out->pitch_words;
-    const uint64_t len = offsets[i + 1] - offsets[i];
-    if (!len) continue;  // an empty stream has no matches (its slots are zeroed above)
-    rx_status s = run(const_cast<rx_program *>(p), d_input + offsets[i], len, 0, 0, offsets[i], nullptr, nullptr,
-                      nullptr, 1, 0, st, &o);
-    if (s != RX_OK) return s;
+    if (out->d_bitstreams) o.d_bitstreams = out->d_bitstreams + a / 32;  // a is a multiple of 1 KiB
+    const void *st_in = i == 0 ? nullptr : p->states[(i + 1) & 1];
+    void *st_out = p->states[i & 1];
+    rx_status r = run(p, (const uint8_t *)p->ring[b] + (a - lo), e - a, a - lo, hi - e, a, st_in, st_out, nullptr,
+                      i == 0 ? 0 : 1, 0, s, &o);
+    if (r != RX_OK) return r;
+    if (cudaEventRecord(p->consumed[b], s) != cudaSuccess) return fail(RX_ECUDA, "event");
   }
   return RX_OK;
 }

@@ -85,3 +85,39 @@ def test_batch_rejects_decreasing_offsets():
     buf = torch.zeros(64, dtype=torch.uint8, device="cuda")
     with pytest.raises(rx.RxError):
         prog.match_batch(buf, [0, 40, 30, 64])
+
+
+def test_batch_many_packets_snort_like():
+    # thousands of packet-sized streams (0-1460 B) of Snort-like payload in ONE
+    # launch sequence, with a Snort-like pattern subset: per-stream counts and
+    # digests equal the oracle run on each stream alone
+    pats = gen.snort_patterns(1000, 2)[0][::5]
+    data = bytes(gen.snort_input(3 << 20, seed=12))
+    rng = np.random.default_rng(12)
+    lens = rng.integers(0, 1461, size=3000)
+    offs = np.concatenate([[0], np.cumsum(lens)]).astype(np.uint64)
+    assert int(offs[-1]) <= len(data)
+    prog = rx.Program(pats)
+    buf = torch.frombuffer(bytearray(data[: int(offs[-1])]), dtype=torch.uint8).cuda()
+    out = prog.match_batch(buf, offs)
+    torch.cuda.synchronize()
+    assert int(out["status"].cpu()[0]) == 0
+    counts = out["counts"].cpu().numpy().view(np.uint64)
+    digests = out["digests"].cpu().numpy().view(np.uint64)
+    regs = [oracle.Regex(p) for p in pats]  # compiled once, run per stream
+    nz = 0
+    for i in range(len(lens)):
+        s = data[int(offs[i]):int(offs[i + 1])]
+        exp_c = np.zeros(len(pats), dtype=np.uint64)
+        exp_d = np.zeros((len(pats), 2), dtype=np.uint64)
+        for r, rg in enumerate(regs):
+            res = rg.run(s, dense=False, positions=True)
+            exp_c[r] = res["count"]
+            for j in res["positions"]:
+                q = int(offs[i]) + int(j)
+                exp_d[r, 0] = (int(exp_d[r, 0]) + oracle.splitmix64(q)) % (1 << 64)
+                exp_d[r, 1] = (int(exp_d[r, 1]) + oracle.splitmix64(q ^ 0x9E3779B97F4A7C15)) % (1 << 64)
+        assert np.array_equal(counts[i], exp_c), i
+        assert np.array_equal(digests[i], exp_d), i
+        nz += int(exp_c.sum())
+    assert nz > 0
