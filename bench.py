@@ -292,6 +292,7 @@ def main():
     ap.add_argument("--interval", type=int, default=0, help="experiment: zero-block guard interval (rx_options)")
     ap.add_argument("--batch", type=int, default=0, help="N3: match N independent packet-sized records (0-1460 B, "
                     "cut from the workload's input) with rx_match_batch, one launch sequence per step")
+    ap.add_argument("--piece-mib", type=int, default=0, help="rx_match_host piece size for e2e (0: library default)")
     ap.add_argument("--split", default="chunk", choices=["chunk", "regex"], help="multi-GPU partition (N>1)")
     ap.add_argument("--ablate", default="", help="comma list of rx flags to set (ablation ladder, DESIGN.md): "
                     "no_prefilter, modeb, no_lockstep, lockstep_round, no_guards, rebalance")
@@ -370,7 +371,7 @@ def main():
             step_device()
             return bout["counts"].to("cpu", non_blocking=False)
         if world == 1:
-            prog.match_host(host, out=out, stream=stream, device=dev)
+            prog.match_host(host, out=out, stream=stream, device=dev, piece_bytes=args.piece_mib << 20)
             return out["counts"].to("cpu", non_blocking=False)
         d_in.copy_(host, non_blocking=True)
         step_device()
@@ -472,7 +473,7 @@ def main():
         line["e2e"] = {"value": total_bytes / (e2e_ms * 1e-3) / 1e9, "unit": "GB/s", "h2d_bytes_per_step": nbytes,
                        "d2h_bytes_per_step": 8 * len(all_pats) * (args.batch or 1),
                        "api": ("H2D copy + rx_match_batch" if args.batch else
-                               "rx_match_host (pinned host input, pipelined 32 MiB pieces)") if world == 1
+                               "rx_match_host (pinned host input, pipelined 64 MiB pieces)") if world == 1
                        else "H2D copy + rx_match_chunk protocol"}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         r, n, dt, thr = oracle_rate(pats, data, target_s=15.0)

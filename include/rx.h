@@ -185,7 +185,7 @@ rx_status rx_match_batch(const rx_program *p, const uint8_t *d_input, const uint
                          void *stream, const rx_output *out);
 
 /* Whole stream from HOST memory, end to end: the input is copied to the
- * device in pieces of piece_bytes (0 = 32 MiB; rounded up to a multiple of
+ * device in pieces of piece_bytes (0 = 64 MiB; rounded up to a multiple of
  * 1 KiB) on an internal copy stream, and piece i is matched with
  * rx_match_chunk while piece i+1 is in flight.  Pieces are matched in order on
  * `stream`, each with rx_max_lookback bytes of the previous piece as its left

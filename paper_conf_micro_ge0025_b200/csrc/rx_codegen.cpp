@@ -284,7 +284,7 @@ struct RegexEmitter {
         std::string t = fresh();
         os << I << "V<" << K << "> " << t << "i;\n";
         for (int i = 0; i < K; ++i) os << I << t << "i.w[" << i << "] = " << W(A, i) << ";\n";
-        os << I << "const V<" << K << "> " << t << "o = rx_lit<" << K << ">(c.lane, c.wb, c.ob, " << t << "i, " << lit_pool << " + "
+        os << I << "const V<" << K << "> " << t << "o = rx_lit<" << K << ">(c.lane, rx_smem_addr(c.wb), rx_smem_addr(c.ob), " << t << "i, " << lit_pool << " + "
            << lit_off[n.cc] << ", " << n.k << ");\n";
         decl(in, nv(id), [&](int i) { return t + "o.w[" + std::to_string(i) + "]"; });
         break;
@@ -362,6 +362,11 @@ struct RegexEmitter {
       for (int i = 0; i < K; ++i) m += (i ? " | " : "") + ("(" + W(R, i) + " & c.cm[" + std::to_string(i) + "])");
       // walk-back runs (mode B) only compute state
       os << I << "if (!c.walk && (c.dense || __any_sync(RX_FULL, (" << m << ") != 0u))) {\n";
+      // counts only: the popcount goes straight into the warp's shared
+      // accumulator (REDUX), no out-of-line call
+      os << I << "  if (c.fast) {\n" << I << "    const u32 cnt_ = __reduce_add_sync(RX_FULL, ";
+      for (int i = 0; i < K; ++i) os << (i ? " + " : "") << "__popc(" << W(R, i) << " & c.cm[" << i << "])";
+      os << ");\n" << I << "    if (lane == 0u) c.acc[" << 3 * out_member[k] << "] += (u64)cnt_;\n" << I << "  } else {\n";
       os << I << "  V<" << K << "> ov;\n";
       os << I << "  u32 cwb = 0u;\n";
       for (int i = 0; i < K; ++i) {
@@ -369,7 +374,7 @@ struct RegexEmitter {
         os << I << "  cwb |= (c.cm[" << i << "] != 0u ? 1u : 0u) << " << i << ";\n";
       }
       os << I << "  rx_emit<" << K << ">(c.o, " << out_member[k] << ", c.lane, c.word0, ov, cwb);\n";
-      os << I << "}\n";
+      os << I << "  }\n" << I << "}\n";
     }
   }
 
@@ -635,18 +640,24 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
      << "  unsigned char *base = rx_warp_smem(warp, " << PER << ");\n"
      << "  RxParams *wp = reinterpret_cast<RxParams *>(base + " << PER - 512 << ");\n"
      << "  const bool batch = pc.batch_off != nullptr;\n"
-     << "  const RxParams &p = batch ? rx_batch_view(pc, wp, seg_in, " << (int)cs.irs.size() << ") : pc;\n"
-     << "  const int seg = batch ? 0 : seg_in;\n"
      << "  u64 *acc = reinterpret_cast<u64 *>(base);\n"
      << "  RxOut *o = reinterpret_cast<RxOut *>(base + " << ACC << ");\n"
      << "  u32 *st = reinterpret_cast<u32 *>(base + " << ACC + OUTB << ");\n"
      << "  unsigned char *lb = base + " << ACC + OUTB + STB << ";\n"
      << "  unsigned char *tb = base + " << ACC + OUTB + STB + LB << ";\n"
      << "  u64 *bar = reinterpret_cast<u64 *>(base + " << ACC + OUTB + STB + LB + TB << ");\n"
-     << "  (void)tb; (void)bar;\n";
+     << "  (void)tb; (void)bar;\n"
+     << "  // one run (a segment of the input), or one run per stream of this\n"
+     << "  // warp's batch segment (one call site of the inlined runner)\n"
+     << "  const long long nrun = batch ? pc.batch_spw : 1;\n"
+     << "  for (long long k = 0; k < nrun; ++k) {\n"
+     << "    const RxParams &p = batch ? rx_batch_view(pc, wp, (long long)seg_in * nrun + k, "
+     << (int)cs.irs.size() << ") : pc;\n"
+     << "    const int seg = batch ? 0 : seg_in;\n"
+     << "    if (batch && rx_batch_skip<RxG" << gi << ">(p)) continue;\n";
   if (cs.use_pf)
-    os << "  if (p.pf_on) { rx_run_segment_pf<RxG" << gi << ">(p, seg, o, acc, st, tb, bar, lb); return; }\n";
-  os << "  rx_run_segment_dense<RxG" << gi << ">(p, seg, o, acc, st, lb);\n}\n";
+    os << "    if (p.pf_on) { rx_run_segment_pf<RxG" << gi << ">(p, seg, o, acc, st, tb, bar, lb); continue; }\n";
+  os << "    rx_run_segment_dense<RxG" << gi << ">(p, seg, o, acc, st, lb);\n  }\n}\n";
   if (g.nslots > 0)
     os << "extern \"C\" __device__ __noinline__ void rx_fix_" << gi << "(int seg) {\n"
        << "  const RxParams &p = rx_cta_params();\n"

@@ -79,6 +79,9 @@ struct Ctx {
   u32 *ob;            // literal-run output scratch, 32*K words (per warp)
   bool walk;          // state-only run (mode-B walk-back): no output
   bool dense;         // dense output requested (mirrors o->want_dense)
+  bool fast;          // counts only (no digests, dense streams or match list) and sign +1: the
+                      // generated epilogue adds the popcount to acc inline, without rx_emit
+  u64 *acc;           // per-warp shared accumulators [NR][3] (== o->acc)
 };
 
 // ---------------------------------------------------------------------------
@@ -212,8 +215,25 @@ __device__ __noinline__ void rx_emit(const RxOut *o, int r, u32 lane, i64 word0,
 // out; the literal holds no 0x00 byte, so positions outside the stream
 // (read as 0) never confirm.
 // ---------------------------------------------------------------------------
+DEV u32 rx_ld_s8(u32 a) {
+  u32 v;
+  asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a));
+  return v;
+}
+DEV u32 rx_ld_s32(u32 a) {
+  u32 v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+  return v;
+}
+DEV void rx_st_s32(u32 a, u32 v) { asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory"); }
+DEV void rx_red_or_s32(u32 a, u32 v) { asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory"); }
+
+// wbs / obs: shared-space addresses of the frame bytes and of the per-warp
+// output words (explicit ld/st/red.shared: handed to an out-of-line function
+// as generic pointers they compiled to generic loads and GPU-scope generic
+// atomics, profiles/r2_ncu_r2n*)
 template <int K>
-__device__ __noinline__ V<K> rx_lit(const u32 lane, const unsigned char *wb, u32 *ob, const V<K> v,
+__device__ __noinline__ V<K> rx_lit(const u32 lane, const u32 wbs, const u32 obs, const V<K> v,
                                     const unsigned char *lit, int n) {
   V<K> r;
   u32 any = 0u;
@@ -225,10 +245,10 @@ __device__ __noinline__ V<K> rx_lit(const u32 lane, const unsigned char *wb, u32
     return r;
   }
 #pragma unroll
-  for (int i = 0; i < K; ++i) ob[lane * K + i] = 0u;
+  for (int i = 0; i < K; ++i) rx_st_s32(obs + 4u * (lane * K + i), 0u);
   __syncwarp();
   const int F = 1024 * K;
-  const unsigned char l0 = lit[0];
+  const u32 l0 = __ldg(lit);
 #pragma unroll
   for (int i = 0; i < K; ++i) {
     u32 b = v.w[i];
@@ -237,15 +257,15 @@ __device__ __noinline__ V<K> rx_lit(const u32 lane, const unsigned char *wb, u32
       b &= b - 1u;
       const int q = (int)((lane * K + i) * 32u) + t;
       const int e = q + n;
-      if (e >= F || wb[q + 1] != l0) continue;
+      if (e >= F || rx_ld_s8(wbs + (u32)q + 1u) != l0) continue;
       int j = 1;
-      while (j < n && wb[q + 1 + j] == lit[j]) ++j;
-      if (j == n) atomicOr(&ob[e >> 5], 1u << (e & 31));
+      while (j < n && rx_ld_s8(wbs + (u32)(q + 1 + j)) == (u32)__ldg(lit + j)) ++j;
+      if (j == n) rx_red_or_s32(obs + 4u * (u32)(e >> 5), 1u << (e & 31));
     }
   }
   __syncwarp();
 #pragma unroll
-  for (int i = 0; i < K; ++i) r.w[i] = ob[lane * K + i];
+  for (int i = 0; i < K; ++i) r.w[i] = rx_ld_s32(obs + 4u * (lane * K + i));
   __syncwarp();
   return r;
 }
@@ -328,10 +348,12 @@ struct RxParams {
   u32 *seg_fix;             // [nseg_max][G][NSMAX]: phase-1 end state of a segment that did not converge
   u32 *seg_nc;              // [nseg_max][G]: that segment did not converge in phase 1
   // rx_match_batch (one launch sequence for all streams): stream s is
-  // in[batch_off[s] .. batch_off[s+1]); pass-1 "segment" s = stream s, whose
-  // warp runs it whole with its own copy of these parameters (rx_batch_view)
+  // in[batch_off[s] .. batch_off[s+1]); pass-1 "segment" j = streams
+  // [j*batch_spw, (j+1)*batch_spw), whose warp runs each whole with its own
+  // copy of these parameters (rx_batch_view)
   const u64 *batch_off;     // device u64[batch_n + 1] (null: not a batch)
   i64 batch_n;
+  i64 batch_spw;            // streams per pass-1 segment (one warp runs them one after the other)
   i64 pf_shift;             // prefilter block coordinates = stream position + pf_shift
 };
 
@@ -378,8 +400,8 @@ DEV const RxParams &rx_batch_view(const RxParams &pc, RxParams *wp, i64 s, int n
     wp->digests = pc.digests ? pc.digests + 2 * ss * nreg : nullptr;
     wp->dense = pc.dense ? pc.dense + (u64)ss * nreg * pc.pitch : nullptr;
     wp->aligned = ((reinterpret_cast<unsigned long long>(wp->in) & 15ull) == 0ull) ? 1 : 0;
-    wp->sw = 1 << 30;
-    wp->nseg_max = 1;
+    wp->nseg_max = 1;  // sw: the host's window count of the longest stream
+    wp->lockstep = 0;  // warps skip streams independently (rx_batch_skip): no CTA barriers
     wp->seg_state = nullptr;
     wp->st_in = nullptr;
     wp->st_out = nullptr;
@@ -503,6 +525,8 @@ template <class G> DEV void rx_ctx_init(const RxParams &p, Ctx<G::K> &c, RxOut *
   c.o = o;
   c.walk = false;
   c.dense = p.dense != nullptr;
+  c.fast = p.dense == nullptr && p.digests == nullptr && p.match_total == nullptr;
+  c.acc = acc;
   c.wb = G::LIT ? lb : nullptr;
   c.ob = G::LIT ? reinterpret_cast<u32 *>(lb + 1024 * G::K) : nullptr;
   if (c.lane == 0) {
@@ -600,6 +624,20 @@ template <class G> DEV u32 rx_run_clusters(u32 rmask, u32 bmc, u32 pendc, u32 la
     r = (G::cmask(ci) & rmask) != 0u || (!(bmc & bit) && (((G::CALWAYS | pendc) & bit) != 0u));
   }
   return __ballot_sync(RX_FULL, r);
+}
+
+// rx_match_batch: a stream none of whose 1 KiB prefilter blocks holds a
+// factor of this group (and the group has no member without a factor) has
+// no match of the group and needs no state: skip it before any setup (most
+// (group, packet) pairs)
+template <class G> DEV bool rx_batch_skip(const RxParams &p) {
+  if (!p.pf_on || G::ALWAYS != 0u) return false;
+  const u32 lane = threadIdx.x & 31u;
+  const u32 *gb = p.pf_gbits + (i64)G::GID * p.pf_ntiles;
+  const i64 b0 = p.pf_shift >> 10, b1 = (p.pf_shift + (p.len > 0 ? p.len : 1) - 1) >> 10;
+  bool hit = false;
+  for (i64 b = b0 + lane; b <= b1; b += 32) hit = hit || ((gb[b >> 5] >> (b & 31)) & 1u);
+  return !__any_sync(RX_FULL, hit);
 }
 
 // ---------------------------------------------------------------------------
@@ -1012,6 +1050,7 @@ DEV void rx_fixup_group(const RxParams &p, RxOut *o, u64 *acc, u32 *sst, unsigne
   auto sstate = [&](const u32 *base, i64 seg) { return base + (seg * G::NG + G::GID) * G::NSMAX; };
   Ctx<K> c;
   rx_ctx_init<G>(p, c, o, acc, lb);
+  c.fast = false;  // the fix-up subtracts (sign -1) and folds match lists: rx_emit only
   // mode-B clusters were exact in pass 1 already: only the others re-run
   const u32 runa = rx_all_clusters<G>() & ~(p.mode == 1 ? rx_mode_b<G>(p, c.lane) : 0u);
   u32 pl[8][K];
