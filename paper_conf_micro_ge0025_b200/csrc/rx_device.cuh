@@ -401,7 +401,6 @@ DEV const RxParams &rx_batch_view(const RxParams &pc, RxParams *wp, i64 s, int n
     wp->dense = pc.dense ? pc.dense + (u64)ss * nreg * pc.pitch : nullptr;
     wp->aligned = ((reinterpret_cast<unsigned long long>(wp->in) & 15ull) == 0ull) ? 1 : 0;
     wp->nseg_max = 1;  // sw: the host's window count of the longest stream
-    wp->lockstep = 0;  // warps skip streams independently (rx_batch_skip): no CTA barriers
     wp->seg_state = nullptr;
     wp->st_in = nullptr;
     wp->st_out = nullptr;
@@ -630,14 +629,19 @@ template <class G> DEV u32 rx_run_clusters(u32 rmask, u32 bmc, u32 pendc, u32 la
 // factor of this group (and the group has no member without a factor) has
 // no match of the group and needs no state: skip it before any setup (most
 // (group, packet) pairs)
-template <class G> DEV bool rx_batch_skip(const RxParams &p) {
-  if (!p.pf_on || G::ALWAYS != 0u) return false;
+// The stream is then run as an empty one (every warp of the CTA still makes
+// the same runner calls: the cluster lockstep's barriers stay matched).
+template <class G> DEV void rx_batch_skip(const RxParams &p, RxParams *wp) {
+  if (!p.pf_on || G::ALWAYS != 0u || p.len <= 0) return;
   const u32 lane = threadIdx.x & 31u;
   const u32 *gb = p.pf_gbits + (i64)G::GID * p.pf_ntiles;
-  const i64 b0 = p.pf_shift >> 10, b1 = (p.pf_shift + (p.len > 0 ? p.len : 1) - 1) >> 10;
+  const i64 b0 = p.pf_shift >> 10, b1 = (p.pf_shift + p.len - 1) >> 10;
   bool hit = false;
   for (i64 b = b0 + lane; b <= b1; b += 32) hit = hit || ((gb[b >> 5] >> (b & 31)) & 1u);
-  return !__any_sync(RX_FULL, hit);
+  if (!__any_sync(RX_FULL, hit)) {
+    if (lane == 0) wp->len = wp->avail_hi = wp->valid_hi = 0;
+    __syncwarp();
+  }
 }
 
 // ---------------------------------------------------------------------------
@@ -1048,6 +1052,14 @@ DEV void rx_fixup_group(const RxParams &p, RxOut *o, u64 *acc, u32 *sst, unsigne
   const i64 nseg = rx_div_up(nwin, p.sw);
   if (p.fix_phase == 1 && (fseg <= 0 || fseg >= nseg)) return;
   auto sstate = [&](const u32 *base, i64 seg) { return base + (seg * G::NG + G::GID) * G::NSMAX; };
+  if (p.mode == 1 && p.fix_phase == 1) {
+    // most segments start from a zero state: nothing to fix, leave before
+    // any setup (phase 1 has a warp for every (group, segment))
+    const u32 *src = sstate(p.seg_state, fseg - 1);
+    bool nz = false;
+    for (int s = (int)(threadIdx.x & 31u); s < NS; s += 32) nz = nz || src[s] != 0u;
+    if (!__any_sync(RX_FULL, nz)) return;
+  }
   Ctx<K> c;
   rx_ctx_init<G>(p, c, o, acc, lb);
   c.fast = false;  // the fix-up subtracts (sign -1) and folds match lists: rx_emit only

@@ -476,6 +476,14 @@ void build_prefilter(CompiledSet &cs) {
   const int nf = (int)cs.factors.size();
   pf.nfactor = nf;
   const Model &mdl = model();
+  // only factors some regex still uses get anchors: output factors are
+  // dropped when mode B is off, and an unused anchor would cost filter hits
+  // and verification for nothing
+  std::vector<char> used(nf, 0);
+  for (auto &rf : cs.rf) {
+    for (int f : rf.first) used[f] = 1;
+    for (int f : rf.out) used[f] = 1;
+  }
   // anchors: per factor the rarest k-gram of narrow consecutive positions
   // (k = 4 preferred), spreading factors over distinct anchors (a shared
   // anchor makes every hit verify every factor that uses it)
@@ -495,6 +503,7 @@ void build_prefilter(CompiledSet &cs) {
     return true;
   };
   for (int f = 0; f < nf; ++f) {
+    if (!used[f]) continue;
     std::set<uint32_t> seen;
     for (int j = 0; j + 4 <= (int)cs.factors[f].win.size(); ++j) {
       uint32_t g;
@@ -511,6 +520,8 @@ void build_prefilter(CompiledSet &cs) {
   };
   for (int f = 0; f < nf; ++f) {
     Factor &F = cs.factors[f];
+    F.grams.clear();
+    if (!used[f]) continue;  // no anchor, no extension entry
     const int L = (int)F.win.size();
     int bk = 0, bj = -1;
     double bs = 1e300;
