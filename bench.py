@@ -292,6 +292,8 @@ def main():
     ap.add_argument("--interval", type=int, default=0, help="experiment: zero-block guard interval (rx_options)")
     ap.add_argument("--batch", type=int, default=0, help="N3: match N independent packet-sized records (0-1460 B, "
                     "cut from the workload's input) with rx_match_batch, one launch sequence per step")
+    ap.add_argument("--outputs", default="counts", choices=["counts", "list"],
+                    help="counts (default) or counts + the compacted match list (rx_output.d_matches)")
     ap.add_argument("--piece-mib", type=int, default=0, help="rx_match_host piece size for e2e (0: library default)")
     ap.add_argument("--split", default="chunk", choices=["chunk", "regex"], help="multi-GPU partition (N>1)")
     ap.add_argument("--ablate", default="", help="comma list of rx flags to set (ablation ladder, DESIGN.md): "
@@ -342,7 +344,10 @@ def main():
     host = torch.from_numpy(np.ascontiguousarray(data)).pin_memory()
     d_in = host.to(dev, non_blocking=False)
     stream = torch.cuda.current_stream(dev)
-    out = prog.alloc_outputs(nbytes, dev, dense=False, digests=False)
+    # the compacted match list (one {regex, position} entry per match end) is
+    # the scalable form of the match-end bitstreams (dense streams: 31 GiB here)
+    list_cap = (64 << 20) if args.outputs == "list" else None
+    out = prog.alloc_outputs(nbytes, dev, dense=False, digests=False, match_cap=list_cap)
 
     def step_device():
         prog.match(d_in, out=out, stream=stream)
@@ -460,7 +465,8 @@ def main():
         "config": {"workload": name, "n_regex": len(all_pats), "input_bytes_per_gpu": nbytes,
                    "parallelism": (f"regex-shard x{world}" if split_regex else f"input-chunk x{world}") if world > 1
                    else "1 GPU",
-                   "groups": prog.n_groups, "outputs": "per-regex counts (dense streams off: 31 GiB at this size)",
+                   "groups": prog.n_groups, "outputs": ("per-regex counts + compacted match list" if args.outputs == "list"
+                               else "per-regex counts (dense streams off: 31 GiB at this size)"),
                    "l2": f"input {nbytes >> 20} MiB per GPU" + (" > 126 MB L2: no flush needed" if nbytes > (126 << 20)
                                                                   else " < L2: L2 flushed between steps"),
                    "prefilter": not args.no_prefilter, "ablate": args.ablate or None, "compile_s": round(compile_s, 1),

@@ -654,7 +654,7 @@ std::string emit_group_unit(CompiledSet &cs, int gi) {
      << "    const RxParams &p = batch ? rx_batch_view(pc, wp, (long long)seg_in * nrun + k, "
      << (int)cs.irs.size() << ") : pc;\n"
      << "    const int seg = batch ? 0 : seg_in;\n"
-     << "    if (batch) rx_batch_skip<RxG" << gi << ">(p, wp);\n";
+     << "    if (batch && !__syncthreads_or(!rx_batch_skip<RxG" << gi << ">(p, wp))) continue;\n";
   if (cs.use_pf)
     os << "    if (p.pf_on) { rx_run_segment_pf<RxG" << gi << ">(p, seg, o, acc, st, tb, bar, lb); continue; }\n";
   os << "    rx_run_segment_dense<RxG" << gi << ">(p, seg, o, acc, st, lb);\n  }\n}\n";

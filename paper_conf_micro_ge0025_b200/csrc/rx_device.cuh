@@ -630,9 +630,11 @@ template <class G> DEV u32 rx_run_clusters(u32 rmask, u32 bmc, u32 pendc, u32 la
 // no match of the group and needs no state: skip it before any setup (most
 // (group, packet) pairs)
 // The stream is then run as an empty one (every warp of the CTA still makes
-// the same runner calls: the cluster lockstep's barriers stay matched).
-template <class G> DEV void rx_batch_skip(const RxParams &p, RxParams *wp) {
-  if (!p.pf_on || G::ALWAYS != 0u || p.len <= 0) return;
+// the same runner calls: the cluster lockstep's barriers stay matched), or --
+// when no warp of the CTA has work for this stream slot -- not at all.
+template <class G> DEV bool rx_batch_skip(const RxParams &p, RxParams *wp) {
+  if (p.len <= 0) return true;
+  if (!p.pf_on || G::ALWAYS != 0u) return false;
   const u32 lane = threadIdx.x & 31u;
   const u32 *gb = p.pf_gbits + (i64)G::GID * p.pf_ntiles;
   const i64 b0 = p.pf_shift >> 10, b1 = (p.pf_shift + p.len - 1) >> 10;
@@ -641,7 +643,9 @@ template <class G> DEV void rx_batch_skip(const RxParams &p, RxParams *wp) {
   if (!__any_sync(RX_FULL, hit)) {
     if (lane == 0) wp->len = wp->avail_hi = wp->valid_hi = 0;
     __syncwarp();
+    return true;
   }
+  return false;
 }
 
 // ---------------------------------------------------------------------------

@@ -14,10 +14,12 @@ for C in dotstar clamav; do
 timeout 900 python bench.py --config $C --steps 5 --warmup 3 --no-cpu-baseline > gpurun_out/bench_${T}_$C.json 2>gpurun_out/bench_${T}_$C.err; echo bench=$?
 tail -1 gpurun_out/bench_${T}_$C.json | cut -c1-400
 done
+timeout 600 python bench.py --outputs list --steps 10 --warmup 3 --no-cpu-baseline > gpurun_out/bench_${T}_list.json 2>gpurun_out/bench_${T}_list.err; echo bench=$?
+tail -1 gpurun_out/bench_${T}_list.json | cut -c1-300
 timeout 600 python bench.py --batch 100000 --steps 10 --warmup 3 --no-cpu-baseline > gpurun_out/bench_${T}_batch.json 2>gpurun_out/bench_${T}_batch.err; echo bench=$?
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 200 --csv --log-file gpurun_out/launches_$T.csv \
   python bench.py --steps 2 --warmup 3 --no-cpu-baseline > gpurun_out/ncu_launch_$T.log 2>&1; echo ncu_launch=$?
-timeout 1500 ncu --set full --clock-control none -k regex:"rx_pass1|rx_prefilter" -s 8 -c 2 \
+timeout 1500 ncu --set full --clock-control none -k regex:"rx_pass1|rx_prefilter" -s 6 -c 2 \
   -o /tmp/prof_$T python bench.py --steps 1 --warmup 3 --no-cpu-baseline > gpurun_out/ncu_full_$T.log 2>&1; echo ncu=$?
 ncu -i /tmp/prof_$T.ncu-rep --page details --csv > gpurun_out/ncu_details_$T.csv 2>&1
 ncu -i /tmp/prof_$T.ncu-rep --page raw --csv > gpurun_out/ncu_raw_$T.csv 2>&1
