@@ -110,3 +110,24 @@ def test_match_batch_validates_offsets_before_any_launch():
     assert st == rx.RX_EINVAL and b"non-decreasing" in p._lib.rx_last_error()
     st = p._lib.rx_match_batch(p._h, None, None, 3, None, ctypes.byref(o))
     assert st == rx.RX_EINVAL
+
+
+def test_match_host_validates_arguments_before_any_copy():
+    # rx_match_host (include/rx.h) rejects null outputs / input and a short
+    # dense pitch before touching the device, so it is checkable on CPU
+    import ctypes
+    import numpy as np
+    p = rx.Program(gen.tiny_patterns())
+    st = p._lib.rx_match_host(p._h, None, 16, 0, None, None)
+    assert st == rx.RX_EINVAL
+    counts = np.zeros(p.n_regex, dtype=np.uint64)
+    o = rx._Output()
+    o.d_counts = counts.ctypes.data
+    st = p._lib.rx_match_host(p._h, None, 16, 0, None, ctypes.byref(o))
+    assert st == rx.RX_EINVAL and b"null input" in p._lib.rx_last_error()
+    buf = np.zeros(4096, dtype=np.uint8)
+    dense = np.zeros(4, dtype=np.uint32)
+    o.d_bitstreams = dense.ctypes.data
+    o.pitch_words = 4
+    st = p._lib.rx_match_host(p._h, buf.ctypes.data, buf.size, 0, None, ctypes.byref(o))
+    assert st == rx.RX_EINVAL and b"pitch_words" in p._lib.rx_last_error()
