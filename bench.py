@@ -111,7 +111,9 @@ class ClockSampler:
 # positions per warp window) measured 24.4 vs 20.2 GB/s at K = 2; the
 # Dotstar-like set is slower at K = 4 (4.1 vs 5.2 GB/s: coarser skipping), so
 # the others keep the compiler's default.
-PROGRAM_OPTS = {"snort": {"words_per_lane": 4}}
+# Round 2: max_regs 168 (12-warp pass-1 CTAs, fewer spills) measured 50.8 vs
+# 47.0 GB/s at 128 (16 warps), profiles/r2_ab_regs.log.
+PROGRAM_OPTS = {"snort": {"words_per_lane": 4, "max_regs": 168}}
 
 WORKLOADS = {
     # name: (pattern builder, input builder(length, rank), default bytes per GPU, description)

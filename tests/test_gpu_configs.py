@@ -45,10 +45,12 @@ def test_config2_snort_like_prefix():
     _parity(pats, gen.snort_input((4 << 20) + 12345, seed=2))
 
 
-def test_config2_snort_like_prefix_bench_k4():
-    # the bench's compile options for this workload (bench.PROGRAM_OPTS: K = 4)
+def test_config2_snort_like_prefix_bench_opts():
+    # the bench's compile options for this workload (bench.PROGRAM_OPTS: K = 4,
+    # 168 registers -> 12-warp pass-1 CTAs)
+    import bench
     pats = gen.snort_patterns(1000, 2)[0]
-    _parity(pats, gen.snort_input((4 << 20) + 12345, seed=2), words_per_lane=4)
+    _parity(pats, gen.snort_input((4 << 20) + 12345, seed=2), **bench.PROGRAM_OPTS["snort"])
 
 
 def test_config3_clamav_brill_prefix():
