@@ -259,9 +259,11 @@ struct rx_program {
   size_t ring_bytes = 0;
   cudaEvent_t copied[kRing] = {nullptr, nullptr, nullptr}, consumed[kRing] = {nullptr, nullptr, nullptr};
   void *states[2] = {nullptr, nullptr};
-  // rx_match_batch: pinned staging of the stream offsets
+  // rx_match_batch: pinned staging of the stream offsets, and the event that
+  // marks the end of its last copy
   void *batch_host = nullptr;
   size_t batch_host_bytes = 0;
+  cudaEvent_t batch_copied = nullptr;
 };
 
 namespace {
@@ -366,6 +368,7 @@ void rx_free(rx_program *p) {
     if (p->states[i]) cudaFree(p->states[i]);
   if (p->copy_stream) cudaStreamDestroy(p->copy_stream);
   if (p->batch_host) cudaFreeHost(p->batch_host);
+  if (p->batch_copied) cudaEventDestroy(p->batch_copied);
   delete p;
 }
 
@@ -1043,23 +1046,24 @@ rx_status rx_match_batch(const rx_program *p, const uint8_t *d_input, const uint
   unsigned long long *h_off = nullptr;
   {
     std::lock_guard<std::mutex> lk(pm->mu);
+    // the previous batch's offsets copy must have read the staging buffer
+    // before it is rewritten (an event, not a stream synchronisation)
+    if (pm->batch_copied) cudaEventSynchronize(pm->batch_copied);
+    else if (cudaEventCreateWithFlags(&pm->batch_copied, cudaEventDisableTiming) != cudaSuccess)
+      return fail(RX_ECUDA, "event");
     if (pm->batch_host_bytes < obytes) {
-      if (pm->batch_host) {
-        cudaStreamSynchronize(st);
-        cudaFreeHost(pm->batch_host);
-      }
+      if (pm->batch_host) cudaFreeHost(pm->batch_host);
       pm->batch_host = nullptr;
       pm->batch_host_bytes = 0;
       if (cudaMallocHost(&pm->batch_host, obytes) != cudaSuccess) return fail(RX_ENOMEM, "batch offsets (host)");
       pm->batch_host_bytes = obytes;
-    } else {
-      cudaStreamSynchronize(st);  // the previous batch's copy has read the staging buffer
     }
     h_off = (unsigned long long *)pm->batch_host;
+    for (uint64_t i = 0; i <= ns; ++i) h_off[i] = offsets[i] - offsets[0];
+    if (cudaMemcpyAsync(d_off, h_off, obytes, cudaMemcpyHostToDevice, st) != cudaSuccess ||
+        cudaEventRecord(pm->batch_copied, st) != cudaSuccess)
+      return fail(RX_ECUDA, "offsets copy");
   }
-  for (uint64_t i = 0; i <= ns; ++i) h_off[i] = offsets[i] - offsets[0];
-  if (cudaMemcpyAsync(d_off, h_off, obytes, cudaMemcpyHostToDevice, st) != cudaSuccess)
-    return fail(RX_ECUDA, "offsets copy");
   BatchArg b{d_off, (long long)ns, (long long)max_len};
   // the streams' match-list positions and digests are relative to d_input
   return run(pm, d_input + offsets[0], total, 0, 0, offsets[0], nullptr, nullptr, nullptr, 1, 0, st, out, &b);

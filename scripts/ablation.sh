@@ -8,7 +8,8 @@
 #   +lock     + cluster lockstep = the default
 #   +modeb    + output-gated clusters (opt-in)            (modeb)
 # sweeps (default path): group size (merge size) 4/16/32, guard interval 1/2/4/8
-# Usage: CONFIGS="snort dotstar" bash scripts/ablation.sh  -> gpurun_out/ablation_<cfg>.jsonl
+# Usage: CONFIGS="snort dotstar" [EXTRA="--length-mib 256"] [RUNGS="base zbs ..."] bash scripts/ablation.sh
+#   -> gpurun_out/ablation_<cfg>.jsonl
 set -x
 mkdir -p gpurun_out
 for C in ${CONFIGS:-snort}; do
@@ -16,19 +17,20 @@ for C in ${CONFIGS:-snort}; do
   : > $OUT
   run() {  # tag, extra bench args
     tag=$1; shift
-    timeout ${RUNG_TIMEOUT:-900} python bench.py --config $C --steps ${STEPS:-3} --warmup 3 --no-cpu-baseline "$@" > /tmp/ab.json 2>/tmp/ab.err
+    timeout ${RUNG_TIMEOUT:-900} python bench.py --config $C --steps ${STEPS:-3} --warmup 3 --no-cpu-baseline ${EXTRA:-} "$@" > /tmp/ab.json 2>/tmp/ab.err
     rc=$?
     echo "{\"rung\": \"$tag\", \"rc\": $rc, \"line\": $(tail -1 /tmp/ab.json | grep '^{' || echo null)}" >> $OUT
     tail -2 /tmp/ab.err
   }
-  run base --ablate no_prefilter,no_guards
-  run zbs --ablate no_prefilter
-  run sr --ablate no_prefilter,rebalance
-  run pf --ablate no_lockstep
-  run lock
-  run modeb --ablate modeb
-  for g in 4 16 32; do run merge$g --group-size $g; done
-  for i in 1 2 4 8; do run interval$i --interval $i; done
+  want() { [ -z "$RUNGS" ] || [[ " $RUNGS " == *" $1 "* ]]; }
+  want base && run base --ablate no_prefilter,no_guards
+  want zbs && run zbs --ablate no_prefilter
+  want sr && run sr --ablate no_prefilter,rebalance
+  want pf && run pf --ablate no_lockstep
+  want lock && run lock
+  want modeb && run modeb --ablate modeb
+  for g in 4 16 32; do want merge$g && run merge$g --group-size $g; done
+  for i in 1 2 4 8; do want interval$i && run interval$i --interval $i; done
   python - "$OUT" <<'PY'
 import json, sys
 for l in open(sys.argv[1]):
