@@ -312,10 +312,18 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # one rank per GPU; RX_DIST_BACKEND=gloo (functional check of the N > 1
+    # path on a one-GPU box: ranks share the GPU, collectives go through the
+    # host, so no kernel waits on another rank's) -- never for a reported number
+    local = local % max(torch.cuda.device_count(), 1)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        backend = os.environ.get("RX_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     split_regex = world > 1 and args.split == "regex"
     # regex split: every rank scans the same input (rank 0's); chunk split:
     # rank r's own chunk of the stream
