@@ -404,9 +404,7 @@ def main():
 
         def step_device():  # noqa: F811
             prog.match(d_in, out=out, stream=stream)
-            full.zero_()
-            full.index_copy_(0, idx, out["counts"])
-            dist.all_reduce(full)
+            parallel.combine_shard_counts(dist, full, idx, out["counts"])
 
     for _ in range(args.warmup):
         step_device()

@@ -45,6 +45,16 @@ def shard_patterns(n: int, world: int, rank: int, costs=None):
     return [i for i in range(n) if owner[i] == rank]
 
 
+def combine_shard_counts(dist, full, idx, local):
+    """Regex sharding: scatter this rank's per-regex results `local` into the
+    zeroed full-length vector `full` at the global regex ids `idx`, then sum
+    over ranks (the shards are disjoint, so the sum is the whole set's)."""
+    full.zero_()
+    full.index_copy_(0, idx, local)
+    all_reduce_sum(dist, full)
+    return full
+
+
 def chunk_bounds(total: int, world: int, rank: int):
     return total * rank // world, total * (rank + 1) // world
 

@@ -146,3 +146,40 @@ def test_chunk_bounds_cover_the_stream():
             cuts = [parallel.chunk_bounds(n, world, r) for r in range(world)]
             assert cuts[0][0] == 0 and cuts[-1][1] == n
             assert all(cuts[i][1] == cuts[i + 1][0] for i in range(world - 1))
+
+
+def _shard_worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        pats = [b"ab", b"abc", b"b", b"zz", b"ca", b"a", b"bca", b"q"]
+        text = b"abcabzzcabcaqab" * 7
+        mine = parallel.shard_patterns(len(pats), world, rank, costs=[float(len(p)) for p in pats])
+        # this rank's "program": overlapping occurrence counts of its own patterns
+        local = torch.tensor([sum(text.startswith(pats[i], k) for k in range(len(text))) for i in mine],
+                             dtype=torch.int64)
+        full = torch.zeros(len(pats), dtype=torch.int64)
+        parallel.combine_shard_counts(dist, full, torch.tensor(mine, dtype=torch.int64), local)
+        q.put((rank, full.tolist()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_regex_shards_combine_to_the_whole_set(world):
+    # bench.py --split regex: disjoint shards, scattered and all-reduced
+    pats = [b"ab", b"abc", b"b", b"zz", b"ca", b"a", b"bca", b"q"]
+    text = b"abcabzzcabcaqab" * 7
+    whole = [sum(text.startswith(p, k) for k in range(len(text))) for p in pats]
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_shard_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=120) for _ in procs]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert all(r[1] == whole for r in res), (whole, res)
