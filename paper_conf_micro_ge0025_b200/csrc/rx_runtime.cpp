@@ -400,13 +400,14 @@ rx_status rx_compile(const char *const *patterns, const size_t *pattern_lens, ui
   auto *p = new rx_program();
   p->n_regex = n_patterns;
   p->flags = o.flags;
-  // pass-1 CTA size: one SM's register file (64 K registers) at max_regs --
-  // 16 warps at 128 registers, 12 at 168, 8 at 255 (rx_options.max_regs)
+  // pass-1 CTA size: one SM's register file (64 K registers) at max_regs
+  // (rx_options.max_regs)
   max_regs = std::max(32, std::min(255, max_regs));
-  // registers are allocated per warp in units of 256 (184 registers take
-  // 6144 per warp, so 11 warps would not fit where 65536 / (32 * 184) says)
-  const int warp_regs = ((32 * max_regs + 255) / 256) * 256;
-  p->pass1_warps = std::max(1, std::min(16, 65536 / warp_regs));
+  // warps are allocated to the SM's four schedulers in groups of four, so a
+  // CTA of 11 warps is budgeted like 12: ptxas caps an entry of 352 threads
+  // at 168 registers, and a group unit compiled for 184 then fails to link
+  // (measured).  Hence 16 warps up to 128 registers, 12 up to 168, else 8.
+  p->pass1_warps = max_regs <= 128 ? 16 : (max_regs <= 168 ? 12 : 8);
   p->cs.pass1_warps = p->pass1_warps;
   p->cs.irs.resize(n_patterns);
   p->cs.factor_of.assign(n_patterns, -1);

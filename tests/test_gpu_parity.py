@@ -201,3 +201,12 @@ def test_bounded_class_repeats_and_literal_runs():
         at = min(at, n - len(s))
         buf[at:at + len(s)] = s
     assert_parity(pats, bytes(buf))
+
+
+@pytest.mark.parametrize("max_regs", [96, 168, 184, 255])
+def test_register_caps_and_cta_sizes(max_regs):
+    # rx_options.max_regs picks the pass-1 CTA size (16 / 12 / 8 warps); every
+    # cap must link (ptxas budgets warps in groups of four) and stay exact
+    pats = gen.tiny_patterns() + [b"x.*y", b"q[^\\n]*z", b"abcdefgh"]
+    data = gen.tiny_input(length=50000, long_chain=2000)
+    assert_parity(pats, data, prog=rx.Program(pats, max_regs=max_regs))
