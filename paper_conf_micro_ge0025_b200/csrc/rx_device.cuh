@@ -1077,10 +1077,22 @@ DEV void rx_fixup_group(const RxParams &p, RxOut *o, u64 *acc, u32 *sst, unsigne
   __syncwarp();
   // re-run windows [w0, w1) with both states (old: the state the applied
   // results assumed, subtracted; tru: the true state, added) until the two
-  // runs' states agree; returns whether they did
-  auto walk = [&](i64 w0, i64 w1) -> bool {
+  // runs' states agree; returns whether they did.  part: run only the
+  // clusters whose state differs between the two runs (clusters are
+  // independent, so an equal state gives equal results: no difference to
+  // apply); their slots then hold 0 in both runs, and `diff` ends as the
+  // clusters that still differ (phase 1 takes the others' end state from
+  // pass 1, which they then follow exactly)
+  u32 diff = runa;
+  auto walk = [&](i64 w0, i64 w1, bool part) -> bool {
     bool conv = rx_state_eq(tru, old, NS, c.lane);
     for (i64 w = w0; w < w1 && !conv; ++w) {
+      if (part) {
+        u32 dm = 0u;
+        for (int s = (int)c.lane; s < NS; s += 32)
+          if (tru[s] != old[s]) dm |= 1u << G::sci(s);
+        diff = __reduce_or_sync(RX_FULL, dm) & runa;
+      }
       const i64 cstart = w * Bw;
       const i64 fword = cstart - Lw;
       c.cw = (u32)((len_words - cstart) < Bw ? (len_words - cstart) : Bw);
@@ -1099,7 +1111,7 @@ DEV void rx_fixup_group(const RxParams &p, RxOut *o, u64 *acc, u32 *sst, unsigne
         for (int j = 0; j < G::NR * K; ++j) fold[j] = 0u;
       __syncwarp();
       rx_state_zero(t1, NS, c.lane);
-      G::body(c, pl, old, t1, runa);
+      G::body(c, pl, old, t1, part ? diff : runa);
       // new run: add, rewrite dense words
       if (c.lane == 0) {
         o->sign = 1ull;
@@ -1108,7 +1120,7 @@ DEV void rx_fixup_group(const RxParams &p, RxOut *o, u64 *acc, u32 *sst, unsigne
       c.dense = p.dense != nullptr;
       __syncwarp();
       rx_state_zero(t2, NS, c.lane);
-      G::body(c, pl, tru, t2, runa);
+      G::body(c, pl, tru, t2, part ? diff : runa);
       __syncwarp();
       rx_state_copy(old, t1, NS, c.lane);
       rx_state_copy(tru, t2, NS, c.lane);
@@ -1130,9 +1142,12 @@ DEV void rx_fixup_group(const RxParams &p, RxOut *o, u64 *acc, u32 *sst, unsigne
     if (rx_state_eq(tru, old, NS, c.lane)) return;
     const i64 w_begin = fseg * p.sw;
     const i64 w_end = w_begin + p.sw < nwin ? w_begin + p.sw : nwin;
-    if (!walk(w_begin, w_end)) {
+    if (!walk(w_begin, w_end, true)) {
+      // the segment's true end state: the walked state of the clusters that
+      // still differ, pass 1's end state for the others
+      const u32 *pe = sstate(p.seg_state, fseg);
       u32 *dst = p.seg_fix + (fseg * G::NG + G::GID) * G::NSMAX;
-      for (int s = (int)c.lane; s < NS; s += 32) dst[s] = tru[s];
+      for (int s = (int)c.lane; s < NS; s += 32) dst[s] = ((diff >> G::sci(s)) & 1u) ? tru[s] : pe[s];
       if (c.lane == 0) p.seg_nc[fseg * G::NG + G::GID] = 1u;
     }
     rx_flush<G>(p, c);
@@ -1154,7 +1169,7 @@ DEV void rx_fixup_group(const RxParams &p, RxOut *o, u64 *acc, u32 *sst, unsigne
       __syncwarp();
       const i64 w_begin = seg * p.sw;
       const i64 w_end = w_begin + p.sw < nwin ? w_begin + p.sw : nwin;
-      if (walk(w_begin, w_end)) {
+      if (walk(w_begin, w_end, false)) {
         // converged: the applied run's end state stands
         const bool nc = p.seg_nc[seg * G::NG + G::GID] != 0u;
         const u32 *e = nc ? sstate(p.seg_fix, seg) : sstate(p.seg_state, seg);
@@ -1174,7 +1189,7 @@ DEV void rx_fixup_group(const RxParams &p, RxOut *o, u64 *acc, u32 *sst, unsigne
     old[s] = p.st_assumed ? p.st_assumed[G::SBASE + s] : 0u;
   }
   __syncwarp();
-  const bool conv = walk(0, nwin);
+  const bool conv = walk(0, nwin, false);
   if (p.st_out && !conv)
     for (int s = (int)c.lane; s < NS; s += 32) p.st_out[G::SBASE + s] = tru[s];
   rx_flush<G>(p, c);
